@@ -1,0 +1,612 @@
+// api.cu — the C ABI of libagraph (include/agraph.h): graph store + inspector (a1), policy and
+// decision maker (a3), and the launch of the device-resident traversal (a2, a4-a7).
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+
+#include "agraph.h"
+#include "common.cuh"
+#include "graph.h"
+#include "traverse.cuh"
+
+using namespace ag;
+
+// ------------------------------------------------------------------------------------------------
+// errors, allocator, launch accounting
+// ------------------------------------------------------------------------------------------------
+static thread_local std::string g_last_error;
+static std::atomic<unsigned long long> g_launches{0};
+
+namespace ag {
+void note_launch(unsigned n) { g_launches += n; }
+
+ag_status set_error(ag_status s, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_last_error = buf;
+    return s;
+}
+
+ag_status cuda_status(cudaError_t e, const char *what) {
+    if (e == cudaSuccess) return AG_OK;
+    cudaGetLastError();
+    if (e == cudaErrorMemoryAllocation) return set_error(AG_ERR_OOM, "%s: %s", what, cudaGetErrorString(e));
+    if (e == cudaErrorNoDevice || e == cudaErrorInsufficientDriver)
+        return set_error(AG_ERR_NO_DEVICE, "%s: %s", what, cudaGetErrorString(e));
+    return set_error(AG_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+static void *(*g_alloc)(size_t, int, void *, void *) = nullptr;
+static void (*g_free)(void *, size_t, int, void *, void *) = nullptr;
+static void *g_alloc_ctx = nullptr;
+
+ag_status dev_alloc(void **p, size_t bytes, int device) {
+    *p = nullptr;
+    if (bytes == 0) bytes = 16;
+    bytes = (bytes + 255) & ~size_t(255);
+    if (g_alloc) {
+        *p = g_alloc(bytes, device, nullptr, g_alloc_ctx);
+        return *p ? AG_OK : set_error(AG_ERR_OOM, "allocator hook returned NULL for %zu bytes", bytes);
+    }
+    return cuda_status(cudaMalloc(p, bytes), "cudaMalloc");
+}
+
+void dev_free(void *p, size_t bytes, int device) {
+    if (!p) return;
+    bytes = (bytes == 0 ? 16 : (bytes + 255) & ~size_t(255));
+    if (g_free) g_free(p, bytes, device, nullptr, g_alloc_ctx);
+    else cudaFree(p);
+}
+
+bool is_device_ptr(const void *p) {
+    if (!p) return false;
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+ag_status check_device(int device, int *num_sms) {
+    int n = 0;
+    cudaError_t e = cudaGetDeviceCount(&n);
+    if (e != cudaSuccess || n == 0) {
+        cudaGetLastError();
+        return set_error(AG_ERR_NO_DEVICE, "no CUDA device available");
+    }
+    if (device < 0 || device >= n) return set_error(AG_ERR_INVALID_ARG, "device %d out of range [0,%d)", device, n);
+    cudaDeviceProp pr;
+    if ((e = cudaGetDeviceProperties(&pr, device)) != cudaSuccess) return cuda_status(e, "cudaGetDeviceProperties");
+    if (pr.major != 10 || pr.minor != 0)
+        return set_error(AG_ERR_NO_DEVICE, "device %d is sm_%d%d; libagraph is built for sm_100a only", device,
+                         pr.major, pr.minor);
+    if (num_sms) *num_sms = pr.multiProcessorCount;
+    return AG_OK;
+}
+}  // namespace ag
+
+// ------------------------------------------------------------------------------------------------
+// graph load kernels: validation + inspector statistics (a1)
+// ------------------------------------------------------------------------------------------------
+struct LoadStats {
+    unsigned int bad;            // bit 0 rp[0], 1 monotone, 2 rp[V], 3 col range, 4 weight range
+    unsigned int min_deg, max_deg, isolated;
+};
+
+__global__ void validate_rows_kernel(const uint64_t *rp, uint32_t V, uint64_t E, LoadStats *st) {
+    uint32_t lmin = 0xFFFFFFFFu, lmax = 0, liso = 0, bad = 0;
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < V; u += gridDim.x * blockDim.x) {
+        uint64_t b = rp[u], e = rp[u + 1];
+        if (e < b) { bad |= 2; continue; }
+        uint64_t d = e - b;
+        uint32_t dd = d > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)d;
+        lmin = min(lmin, dd);
+        lmax = max(lmax, dd);
+        liso += (d == 0);
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        if (rp[0] != 0) bad |= 1;
+        if (rp[V] != E) bad |= 4;
+    }
+    lmin = warp_min(lmin);
+    for (int o = 16; o > 0; o >>= 1) lmax = max(lmax, __shfl_xor_sync(0xffffffffu, lmax, o));
+    liso = warp_sum(liso);
+    bad |= __reduce_or_sync(0xffffffffu, bad);
+    if ((threadIdx.x & 31) == 0) {
+        atomicMin(&st->min_deg, lmin);
+        atomicMax(&st->max_deg, lmax);
+        if (liso) atomicAdd(&st->isolated, liso);
+        if (bad) atomicOr(&st->bad, bad);
+    }
+}
+
+__global__ void validate_edges_kernel(const uint32_t *col, const uint32_t *w, uint64_t E, uint32_t V, LoadStats *st) {
+    unsigned bad = 0;
+    for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < E; e += (uint64_t)gridDim.x * blockDim.x) {
+        if (col[e] >= V) bad |= 8;
+        if (w) {
+            uint32_t x = w[e];
+            if (x == 0 || x >= 0x80000000u) bad |= 16;
+        }
+    }
+    bad = __reduce_or_sync(0xffffffffu, bad);
+    if ((threadIdx.x & 31) == 0 && bad) atomicOr(&st->bad, bad);
+}
+
+__global__ void narrow_offsets_kernel(const uint64_t *rp, uint32_t *rp32, uint32_t n) {
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+        rp32[i] = (uint32_t)rp[i];
+}
+
+// V_r and E_r of a result array (stats only; not in the timed path)
+template <typename Off>
+__global__ void reached_kernel(const uint32_t *out, const Off *rp, uint32_t V, unsigned long long *acc) {
+    unsigned long long a = 0, b = 0;
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x)
+        if (out[v] != INF) { a += 1; b += (unsigned long long)(rp[v + 1] - rp[v]); }
+    a = warp_sum(a);
+    b = warp_sum(b);
+    if ((threadIdx.x & 31) == 0 && (a | b)) { atomicAdd(&acc[0], a); atomicAdd(&acc[1], b); }
+}
+
+// exact overflow test after a flagged SSSP: a reachable vertex left at INF behind a finite one
+template <typename Off>
+__global__ void overflow_check_kernel(const uint32_t *dist, const Off *rp, const uint32_t *col, uint32_t V,
+                                      unsigned *flag) {
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < V; u += gridDim.x * blockDim.x) {
+        if (dist[u] == INF) continue;
+        for (Off e = rp[u]; e < rp[u + 1]; ++e)
+            if (dist[col[e]] == INF) { *flag = 1; return; }
+    }
+}
+
+// ------------------------------------------------------------------------------------------------
+// graph handle helpers
+// ------------------------------------------------------------------------------------------------
+namespace ag {
+
+static ag_status ensure_scratch(ag_graph_s *g, bool sssp) {
+    const size_t V = g->V, nw = g->nwords;
+    ag_status s;
+#define ALLOC(ptr, bytes)                                                          \
+    if (!(ptr)) {                                                                  \
+        if ((s = dev_alloc((void **)&(ptr), (bytes), g->device)) != AG_OK) return s; \
+        g->scratch_bytes += (bytes);                                               \
+    }
+    ALLOC(g->d_ctl, sizeof(Ctl));
+    if (!g->ctl_init) {
+        cudaMemset(g->d_ctl, 0, sizeof(Ctl));
+        g->ctl_init = true;
+    }
+    for (int i = 0; i < 3; ++i) { ALLOC(g->d_bm[i], nw * 4 + 128); }
+    for (int i = 0; i < 3; ++i) { ALLOC(g->d_q[i], V * 4 + 128); }
+    ALLOC(g->d_vis, nw * 4 + 128);
+    ALLOC(g->d_hub, (size_t)g->hub_cap * 16);
+    ALLOC(g->d_acc, 64);
+    if (sssp) { ALLOC(g->d_P, V * 8 + 128); }
+#undef ALLOC
+    return AG_OK;
+}
+
+static ag_status ensure_buf(ag_graph_s *g, uint32_t **p, size_t *have, size_t bytes) {
+    if (*have >= bytes && *p) return AG_OK;
+    if (*p) dev_free(*p, *have, g->device);
+    *p = nullptr;
+    *have = 0;
+    ag_status s = dev_alloc((void **)p, bytes, g->device);
+    if (s == AG_OK) *have = bytes;
+    return s;
+}
+
+DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
+    DevPolicy d;
+    memset(&d, 0, sizeof d);
+    d.kind = p.kind;
+    d.force_map = p.mapping;
+    d.force_ws = p.workset;
+    d.t1 = p.t1_avg_degree;
+    d.t2 = p.t2_ws;
+    d.t3 = ((uint64_t)g.V * p.t3_ppm + 999999ull) / 1000000ull;
+    d.sample_every = p.sample_every ? p.sample_every : 1;
+    d.delta = p.delta ? p.delta : 1;
+    uint32_t grp = p.cta_group;
+    if (grp == 0) {  // multiple of 32 closest to the average out-degree, ties up (26.s28, R16)
+        uint64_t k = g.V ? (2 * g.E + 32ull * g.V) / (64ull * g.V) : 1;
+        grp = (uint32_t)(32 * (k < 1 ? 1 : k));
+    }
+    grp = grp < 32 ? 32 : grp;
+    grp = grp > (uint32_t)BS ? (uint32_t)BS : grp;
+    grp &= ~31u;
+    d.cta_group = grp;
+    d.V = g.V;
+    d.E = g.E;
+    return d;
+}
+
+ag_status check_policy(const ag_policy *p) {
+    if (p->struct_size != sizeof(ag_policy)) return set_error(AG_ERR_INVALID_ARG, "ag_policy.struct_size mismatch");
+    if (p->order > AG_ORDERED || p->mapping > AG_MAP_HYBRID || p->workset > AG_WS_QUEUE || p->kind > AG_POLICY_TUNED)
+        return set_error(AG_ERR_INVALID_ARG, "ag_policy field out of range");
+    if (p->cta_group % 32) return set_error(AG_ERR_INVALID_ARG, "cta_group must be a multiple of 32");
+    if (p->delta == 0 || p->delta >= 0x80000000u) return set_error(AG_ERR_INVALID_ARG, "delta must be in [1, 2^31)");
+    return AG_OK;
+}
+
+}  // namespace ag
+
+// ------------------------------------------------------------------------------------------------
+// traversal launch
+// ------------------------------------------------------------------------------------------------
+template <int ALG, int ORD, typename Off>
+static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t st) {
+    auto fn = traverse_kernel<ALG, ORD, Off>;
+    int occ = 0;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, BS, 0);
+    if (e != cudaSuccess || occ < 1) return cuda_status(e == cudaSuccess ? cudaErrorLaunchOutOfResources : e, "occupancy");
+    a.nblocks = (uint32_t)(occ * g->num_sms);
+    void *args[] = {(void *)&a};
+    e = cudaLaunchCooperativeKernel((const void *)fn, dim3(a.nblocks), dim3(BS), args, 0, st);
+    note_launch(1);
+    return cuda_status(e, "traverse launch");
+}
+
+template <typename Off>
+static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, uint32_t *parents,
+                           const ag_policy *pin, ag_run_stats *stats, cudaStream_t st) {
+    ag_policy pol;
+    if (pin) {
+        pol = *pin;
+    } else {
+        ag_policy_default(&pol, g->device);
+    }
+    ag_status s = check_policy(&pol);
+    if (s != AG_OK) return s;
+    if (stats && stats->struct_size != sizeof(ag_run_stats))
+        return set_error(AG_ERR_INVALID_ARG, "ag_run_stats.struct_size mismatch");
+    cudaSetDevice(g->device);
+    if ((s = ensure_scratch(g, alg == ALG_SSSP)) != AG_OK) return s;
+
+    const bool out_dev = is_device_ptr(out);
+    const bool par_dev = parents ? is_device_ptr(parents) : true;
+    const bool sync = stats != nullptr || !out_dev || !par_dev;
+    const size_t vbytes = (size_t)g->V * 4 + 128;
+    uint32_t *d_out = out, *d_par = parents;
+    if (!out_dev) {
+        if ((s = ensure_buf(g, &g->d_out_tmp, &g->out_tmp_bytes, vbytes)) != AG_OK) return s;
+        d_out = g->d_out_tmp;
+    }
+    if (parents && !par_dev) {
+        if ((s = ensure_buf(g, &g->d_par_tmp, &g->par_tmp_bytes, vbytes)) != AG_OK) return s;
+        d_par = g->d_par_tmp;
+    }
+    uint32_t tcap = (stats && (stats->trace_ws || stats->trace_edges || stats->trace_variant)) ? stats->trace_cap : 0;
+    if (tcap) {
+        size_t need = (size_t)tcap * 16;
+        if ((s = ensure_buf(g, &g->d_trace, &g->trace_bytes, need)) != AG_OK) return s;
+    }
+
+    TravArgs<Off> a;
+    memset(&a, 0, sizeof a);
+    a.rp = (const Off *)g->d_rp;
+    a.col = g->d_col;
+    a.w = g->d_w;
+    a.V = g->V;
+    a.nwords = g->nwords;
+    a.P = g->d_P;
+    a.vis = g->d_vis;
+    for (int i = 0; i < 3; ++i) { a.bm[i] = g->d_bm[i]; a.q[i] = g->d_q[i]; }
+    a.hub = g->d_hub;
+    a.hub_cap = g->hub_cap;
+    a.ctl = (Ctl *)g->d_ctl;
+    if (alg == ALG_BFS) {
+        a.level = d_out;
+        a.parent = d_par;
+    } else {
+        a.dist_out = d_out;
+        a.parent_out = d_par;
+    }
+    if (tcap) {
+        uint8_t *base = (uint8_t *)g->d_trace;
+        a.trace_edges = (unsigned long long *)base;
+        a.trace_ws = (uint32_t *)(base + (size_t)tcap * 8);
+        a.trace_var = base + (size_t)tcap * 12;
+        a.trace_cap = tcap;
+    }
+    a.pol = resolve_policy(pol, *g);
+    a.src = src;
+    a.epoch = ++g->epoch;
+    a.max_iters = alg == ALG_BFS ? g->V + 2 : 4u * g->V + 64u;
+    if (a.max_iters < g->V) a.max_iters = 0xFFFFFFF0u;
+    a.has_hubs = g->info.max_deg >= HUB_DEG;
+
+    if (stats) {
+        cudaEventRecord(g->ev[0], st);
+    }
+    if (alg == ALG_BFS) {
+        s = (pol.order == AG_ORDERED) ? launch_traverse<ALG_BFS, ORD_O, Off>(g, a, st)
+                                      : launch_traverse<ALG_BFS, ORD_U, Off>(g, a, st);
+    } else {
+        s = (pol.order == AG_ORDERED) ? launch_traverse<ALG_SSSP, ORD_O, Off>(g, a, st)
+                                      : launch_traverse<ALG_SSSP, ORD_U, Off>(g, a, st);
+    }
+    if (s != AG_OK) return s;
+    if (stats) cudaEventRecord(g->ev[1], st);
+    g->last_stream = st;
+    g->last_alg = alg;
+    g->last_out = d_out;
+    g->pending_check = true;
+
+    if (!out_dev) cudaMemcpyAsync(out, d_out, (size_t)g->V * 4, cudaMemcpyDeviceToHost, st);
+    if (parents && !par_dev) cudaMemcpyAsync(parents, d_par, (size_t)g->V * 4, cudaMemcpyDeviceToHost, st);
+    if (!sync) return cuda_status(cudaGetLastError(), "enqueue");
+
+    if (stats) {
+        cudaMemsetAsync(g->d_acc, 0, 16, st);
+        reached_kernel<Off><<<g->num_sms * 4, 256, 0, st>>>(d_out, (const Off *)g->d_rp, g->V,
+                                                             (unsigned long long *)g->d_acc);
+        note_launch(1);
+    }
+    cudaError_t e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_status(e, "traversal");
+    s = ag_graph_check(g);
+    if (s != AG_OK && s != AG_ERR_OVERFLOW) return s;
+    if (stats) {
+        Ctl c;
+        cudaMemcpy(&c, g->d_ctl, sizeof c, cudaMemcpyDeviceToHost);
+        unsigned long long acc[2];
+        cudaMemcpy(acc, g->d_acc, 16, cudaMemcpyDeviceToHost);
+        stats->iterations = c.iterations;
+        stats->vertices_expanded = c.vexp;
+        stats->edges_inspected = c.eexp;
+        stats->reached = acc[0];
+        stats->reached_edges = acc[1];
+        float ms = 0;
+        cudaEventElapsedTime(&ms, g->ev[0], g->ev[1]);
+        stats->device_ms = ms;
+        uint32_t n = c.iterations < tcap ? c.iterations : tcap;
+        stats->trace_len = n;
+        if (n) {
+            uint8_t *base = (uint8_t *)g->d_trace;
+            if (stats->trace_edges) cudaMemcpy(stats->trace_edges, base, (size_t)n * 8, cudaMemcpyDeviceToHost);
+            if (stats->trace_ws) cudaMemcpy(stats->trace_ws, base + (size_t)tcap * 8, (size_t)n * 4, cudaMemcpyDeviceToHost);
+            if (stats->trace_variant) cudaMemcpy(stats->trace_variant, base + (size_t)tcap * 12, n, cudaMemcpyDeviceToHost);
+        }
+        e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_status(e, "stats");
+        if (c.aborted) return set_error(AG_ERR_CUDA, "traversal aborted (code %u)", c.aborted);
+    }
+    return s;
+}
+
+// ------------------------------------------------------------------------------------------------
+// C ABI
+// ------------------------------------------------------------------------------------------------
+extern "C" {
+
+uint32_t ag_abi_version(void) { return AG_ABI_VERSION; }
+uint64_t ag_kernel_launches(void) { return g_launches.load(); }
+const char *ag_last_error(void) { return g_last_error.c_str(); }
+
+const char *ag_status_string(ag_status s) {
+    switch (s) {
+        case AG_OK: return "AG_OK";
+        case AG_ERR_INVALID_ARG: return "AG_ERR_INVALID_ARG";
+        case AG_ERR_BAD_CSR: return "AG_ERR_BAD_CSR";
+        case AG_ERR_SRC_RANGE: return "AG_ERR_SRC_RANGE";
+        case AG_ERR_NO_WEIGHTS: return "AG_ERR_NO_WEIGHTS";
+        case AG_ERR_OVERFLOW: return "AG_ERR_OVERFLOW";
+        case AG_ERR_OOM: return "AG_ERR_OOM";
+        case AG_ERR_CUDA: return "AG_ERR_CUDA";
+        case AG_ERR_NCCL: return "AG_ERR_NCCL";
+        case AG_ERR_UNSUPPORTED: return "AG_ERR_UNSUPPORTED";
+        case AG_ERR_NO_DEVICE: return "AG_ERR_NO_DEVICE";
+    }
+    return "AG_ERR_?";
+}
+
+ag_status ag_set_allocator(void *(*alloc)(size_t, int, void *, void *), void (*free_)(void *, size_t, int, void *, void *),
+                           void *ctx) {
+    if ((alloc == nullptr) != (free_ == nullptr)) return set_error(AG_ERR_INVALID_ARG, "alloc and free must both be set");
+    g_alloc = alloc;
+    g_free = free_;
+    g_alloc_ctx = ctx;
+    return AG_OK;
+}
+
+ag_status ag_policy_default(ag_policy *p, int device) {
+    if (!p) return set_error(AG_ERR_INVALID_ARG, "policy is NULL");
+    int sms = 0;
+    ag_status s = check_device(device, &sms);
+    if (s != AG_OK) return s;
+    memset(p, 0, sizeof *p);
+    p->struct_size = sizeof(ag_policy);
+    p->order = AG_UNORDERED;
+    p->mapping = AG_MAP_AUTO;
+    p->workset = AG_WS_AUTO;
+    p->kind = AG_POLICY_TUNED;
+    p->t1_avg_degree = 32;
+    p->thread_tpb = 192;
+    p->t2_ws = 192ull * (uint64_t)sms;
+    p->t3_ppm = 15625;
+    p->sample_every = 1;
+    p->delta = 1;
+    p->cta_group = 0;
+    return AG_OK;
+}
+
+uint8_t ag_select(const ag_policy *p, const ag_graph_info *gi, uint64_t ws_size, uint64_t ws_edges) {
+    if (!p || !gi || check_policy(p) != AG_OK) return 0;
+    ag_graph_s tmp;
+    tmp.V = gi->num_vertices;
+    tmp.E = gi->num_edges;
+    DevPolicy d = resolve_policy(*p, tmp);
+    return select_variant(d, ws_size, ws_edges);
+}
+
+ag_status ag_graph_load_csr(uint32_t V, uint64_t E, const uint64_t *row_ptr, const uint32_t *col_idx,
+                            const uint32_t *weights, int device, ag_graph *out) {
+    if (!out || !row_ptr || (!col_idx && E > 0)) return set_error(AG_ERR_INVALID_ARG, "NULL argument");
+    *out = nullptr;
+    if (V == 0 || V >= 0xFFFFFFFFu) return set_error(AG_ERR_BAD_CSR, "V must be in [1, 2^32-1)");
+    int sms = 0;
+    ag_status s = check_device(device, &sms);
+    if (s != AG_OK) return s;
+    cudaSetDevice(device);
+    ag_graph_s *g = new ag_graph_s();
+    g->device = device;
+    g->V = V;
+    g->E = E;
+    g->num_sms = sms;
+    g->nwords = (V + 31) / 32;
+    g->offs32 = E < 0xFFFFFFFFull;
+    g->hub_cap = (uint32_t)((E / HUB_CHUNK + E / HUB_DEG + 16) > 0xFFFFFFF0ull ? 0xFFFFFFF0ull
+                                                                            : (E / HUB_CHUNK + E / HUB_DEG + 16));
+    cudaEventCreate(&g->ev[0]);
+    cudaEventCreate(&g->ev[1]);
+    auto fail = [&](ag_status st) { ag_graph_free(g); return st; };
+
+    uint64_t *rp64 = nullptr;
+    LoadStats *dst = nullptr;
+    if ((s = dev_alloc((void **)&rp64, (size_t)(V + 1) * 8, device)) != AG_OK) return fail(s);
+    if ((s = dev_alloc((void **)&g->d_col, E * 4 + 128, device)) != AG_OK) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(s); }
+    g->col_bytes = E * 4 + 128;
+    if (weights) {
+        if ((s = dev_alloc((void **)&g->d_w, E * 4 + 128, device)) != AG_OK) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(s); }
+        g->w_bytes = E * 4 + 128;
+    }
+    if ((s = dev_alloc((void **)&dst, sizeof(LoadStats), device)) != AG_OK) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(s); }
+    cudaError_t e = cudaMemcpy(rp64, row_ptr, (size_t)(V + 1) * 8, cudaMemcpyDefault);
+    if (e == cudaSuccess && E) e = cudaMemcpy(g->d_col, col_idx, E * 4, cudaMemcpyDefault);
+    if (e == cudaSuccess && E && weights) e = cudaMemcpy(g->d_w, weights, E * 4, cudaMemcpyDefault);
+    LoadStats hs = {0, 0xFFFFFFFFu, 0, 0};
+    if (e == cudaSuccess) e = cudaMemcpy(dst, &hs, sizeof hs, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) {
+        validate_rows_kernel<<<sms * 8, 256>>>(rp64, V, E, dst);
+        if (E) validate_edges_kernel<<<sms * 8, 256>>>(g->d_col, weights ? g->d_w : nullptr, E, V, dst);
+        note_launch(E ? 2 : 1);
+        e = cudaMemcpy(&hs, dst, sizeof hs, cudaMemcpyDeviceToHost);
+    }
+    dev_free(dst, sizeof(LoadStats), device);
+    if (e != cudaSuccess) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(cuda_status(e, "graph load")); }
+    if (hs.bad) {
+        dev_free(rp64, (size_t)(V + 1) * 8, device);
+        return fail(set_error(AG_ERR_BAD_CSR, "invalid CSR (%s%s%s%s%s)", hs.bad & 1 ? "row_ptr[0]!=0 " : "",
+                              hs.bad & 2 ? "non-monotone row_ptr " : "", hs.bad & 4 ? "row_ptr[V]!=E " : "",
+                              hs.bad & 8 ? "col>=V " : "", hs.bad & 16 ? "weight not in [1,2^31) " : ""));
+    }
+    if (g->offs32) {
+        uint32_t *rp32 = nullptr;
+        if ((s = dev_alloc((void **)&rp32, (size_t)(V + 1) * 4 + 128, device)) != AG_OK) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(s); }
+        narrow_offsets_kernel<<<sms * 8, 256>>>(rp64, rp32, V + 1);
+        note_launch(1);
+        e = cudaDeviceSynchronize();
+        dev_free(rp64, (size_t)(V + 1) * 8, device);
+        if (e != cudaSuccess) { dev_free(rp32, (size_t)(V + 1) * 4 + 128, device); return fail(cuda_status(e, "narrow")); }
+        g->d_rp = rp32;
+        g->rp_bytes = (size_t)(V + 1) * 4 + 128;
+    } else {
+        g->d_rp = rp64;
+        g->rp_bytes = (size_t)(V + 1) * 8;
+    }
+    g->info.num_vertices = V;
+    g->info.num_edges = E;
+    g->info.deg_sum = E;
+    g->info.min_deg = hs.min_deg == 0xFFFFFFFFu ? 0 : hs.min_deg;
+    g->info.max_deg = hs.max_deg;
+    g->info.isolated = hs.isolated;
+    g->info.weighted = weights ? 1 : 0;
+    g->info.device = device;
+    g->info.num_sms = sms;
+    g->info.offset_bytes = g->offs32 ? 4 : 8;
+    *out = g;
+    return AG_OK;
+}
+
+ag_status ag_graph_info_get(ag_graph g, ag_graph_info *out) {
+    if (!g || !out) return set_error(AG_ERR_INVALID_ARG, "NULL argument");
+    *out = g->info;
+    return AG_OK;
+}
+
+ag_status ag_graph_free(ag_graph g) {
+    if (!g) return set_error(AG_ERR_INVALID_ARG, "NULL graph");
+    cudaSetDevice(g->device);
+    if (g->last_stream || g->pending_check) cudaDeviceSynchronize();
+    dev_free(g->d_rp, g->rp_bytes, g->device);
+    dev_free(g->d_col, g->col_bytes, g->device);
+    dev_free(g->d_w, g->w_bytes, g->device);
+    const size_t V = g->V, nw = g->nwords;
+    dev_free(g->d_ctl, sizeof(Ctl), g->device);
+    for (int i = 0; i < 3; ++i) { dev_free(g->d_bm[i], nw * 4 + 128, g->device); dev_free(g->d_q[i], V * 4 + 128, g->device); }
+    dev_free(g->d_vis, nw * 4 + 128, g->device);
+    dev_free(g->d_hub, (size_t)g->hub_cap * 16, g->device);
+    dev_free(g->d_acc, 64, g->device);
+    dev_free(g->d_P, V * 8 + 128, g->device);
+    dev_free(g->d_out_tmp, g->out_tmp_bytes, g->device);
+    dev_free(g->d_par_tmp, g->par_tmp_bytes, g->device);
+    dev_free(g->d_trace, g->trace_bytes, g->device);
+    if (g->ev[0]) cudaEventDestroy(g->ev[0]);
+    if (g->ev[1]) cudaEventDestroy(g->ev[1]);
+    ag::dist_graph_release(g);
+    delete g;
+    return AG_OK;
+}
+
+ag_status ag_graph_check(ag_graph g) {
+    if (!g) return set_error(AG_ERR_INVALID_ARG, "NULL graph");
+    if (!g->pending_check) return AG_OK;
+    cudaSetDevice(g->device);
+    cudaError_t e = cudaStreamSynchronize(g->last_stream);
+    if (e != cudaSuccess) return cuda_status(e, "traversal");
+    g->pending_check = false;
+    Ctl c;
+    e = cudaMemcpy(&c, g->d_ctl, sizeof c, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return cuda_status(e, "ctl");
+    if (c.aborted) return set_error(AG_ERR_CUDA, "traversal aborted (code %u)", c.aborted);
+    if (g->last_alg == ALG_SSSP && c.overflow) {
+        unsigned *flag = (unsigned *)g->d_acc;
+        cudaMemset(flag, 0, 4);
+        if (g->offs32)
+            overflow_check_kernel<uint32_t><<<g->num_sms * 4, 256>>>(g->last_out, (const uint32_t *)g->d_rp, g->d_col, g->V, flag);
+        else
+            overflow_check_kernel<unsigned long long><<<g->num_sms * 4, 256>>>(g->last_out, (const unsigned long long *)g->d_rp, g->d_col, g->V, flag);
+        note_launch(1);
+        unsigned h = 0;
+        e = cudaMemcpy(&h, flag, 4, cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) return cuda_status(e, "overflow check");
+        if (h) return set_error(AG_ERR_OVERFLOW, "a finite distance exceeds 0xFFFFFFFE");
+    }
+    return AG_OK;
+}
+
+static ag_status query(ag_graph g, int alg, uint32_t src, uint32_t *out, uint32_t *parents, const ag_policy *p,
+                       ag_run_stats *stats, void *stream) {
+    if (!g || !out) return set_error(AG_ERR_INVALID_ARG, "NULL argument");
+    if (src >= g->V) return set_error(AG_ERR_SRC_RANGE, "src %u >= V %u", src, g->V);
+    if (alg == ALG_SSSP && !g->d_w) return set_error(AG_ERR_NO_WEIGHTS, "graph was loaded without weights");
+    if (g->dist) return set_error(AG_ERR_INVALID_ARG, "distributed graph: use ag_dist_bfs");
+    cudaStream_t st = (cudaStream_t)stream;
+    return g->offs32 ? run_query<uint32_t>(g, alg, src, out, parents, p, stats, st)
+                     : run_query<unsigned long long>(g, alg, src, out, parents, p, stats, st);
+}
+
+ag_status ag_bfs(ag_graph g, uint32_t src, uint32_t *levels, uint32_t *parents, const ag_policy *policy,
+                 ag_run_stats *stats, void *stream) {
+    return query(g, ALG_BFS, src, levels, parents, policy, stats, stream);
+}
+
+ag_status ag_sssp(ag_graph g, uint32_t src, uint32_t *dist, uint32_t *parents, const ag_policy *policy,
+                  ag_run_stats *stats, void *stream) {
+    return query(g, ALG_SSSP, src, dist, parents, policy, stats, stream);
+}
+
+}  // extern "C"

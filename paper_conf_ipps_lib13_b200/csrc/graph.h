@@ -1,0 +1,67 @@
+// graph.h — the library-owned graph handle (device CSR + per-handle traversal scratch).
+//
+// HBM layout: row offsets u32 when E < 2^32 (else u64), col_idx u32, weights u32,
+// all cudaMalloc'd (256-B aligned).  Scratch: 3 frontier bitmaps (V/8 B each), 3 queues (4V B
+// each), visited bitmap (V/8 B), packed SSSP state (8V B), hub-chunk task ring, control block.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "agraph.h"
+
+struct ag_dist_part;  // multi-GPU partition data (dist.cu)
+
+struct ag_graph_s {
+    int device = 0;
+    uint32_t V = 0;
+    uint64_t E = 0;
+    uint32_t nwords = 0;
+    int num_sms = 0;
+    bool offs32 = true;
+    ag_graph_info info{};
+    // CSR
+    void *d_rp = nullptr;
+    size_t rp_bytes = 0;
+    uint32_t *d_col = nullptr;
+    size_t col_bytes = 0;
+    uint32_t *d_w = nullptr;
+    size_t w_bytes = 0;
+    // scratch
+    void *d_ctl = nullptr;
+    bool ctl_init = false;
+    uint32_t *d_bm[3] = {nullptr, nullptr, nullptr};
+    uint32_t *d_q[3] = {nullptr, nullptr, nullptr};
+    uint32_t *d_vis = nullptr;
+    uint32_t *d_hub = nullptr;
+    uint32_t hub_cap = 0;
+    unsigned long long *d_P = nullptr;
+    void *d_acc = nullptr;
+    uint32_t *d_out_tmp = nullptr;
+    size_t out_tmp_bytes = 0;
+    uint32_t *d_par_tmp = nullptr;
+    size_t par_tmp_bytes = 0;
+    uint32_t *d_trace = nullptr;
+    size_t trace_bytes = 0;
+    size_t scratch_bytes = 0;
+    cudaEvent_t ev[2] = {nullptr, nullptr};
+    uint32_t epoch = 0;
+    // deferred status of the last enqueued traversal
+    cudaStream_t last_stream = nullptr;
+    int last_alg = 0;
+    uint32_t *last_out = nullptr;
+    bool pending_check = false;
+    // multi-GPU
+    ag_dist_part *dist = nullptr;
+};
+
+namespace ag {
+ag_status set_error(ag_status s, const char *fmt, ...);
+ag_status cuda_status(cudaError_t e, const char *what);
+ag_status dev_alloc(void **p, size_t bytes, int device);
+void dev_free(void *p, size_t bytes, int device);
+bool is_device_ptr(const void *p);
+ag_status check_device(int device, int *num_sms);
+void note_launch(unsigned n);
+void dist_graph_release(ag_graph_s *g);
+}  // namespace ag

@@ -1,0 +1,266 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, bit-exact (-m gpu).
+
+Levels and distances are unique and compared element by element (memcmp); parents are
+legitimately nondeterministic and are checked with the oracle's certificate validator
+(SURVEY.md §8(c)).  Every variant of the three axes is exercised: {ordered, unordered} x
+{thread, warp, CTA, hybrid} x {bitmap, queue}, plus the adaptive selector (paper and tuned).
+"""
+import numpy as np
+import pytest
+
+import aggen
+import oracle
+from oracle import selector
+
+pytestmark = pytest.mark.gpu
+
+A = None
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    global A
+    from paper_conf_ipps_lib13_b200 import agraph, build
+    build.build()
+    A = agraph
+    yield
+
+
+INF = oracle.INF
+MAPS = [1, 2, 3, 4]            # T, W, B(CTA), H
+WSS = [1, 2]                   # BM, QU
+
+
+def pol(order=0, mapping=0, workset=0, kind=1, **kw):
+    p = A.policy_default(0)
+    p.order, p.mapping, p.workset, p.kind = order, mapping, workset, kind
+    for k, v in kw.items():
+        setattr(p, k, v)
+    return p
+
+
+def all_policies():
+    out = []
+    for order in (0, 1):
+        for m in MAPS:
+            for w in WSS:
+                out.append(pol(order, m, w))
+        out.append(pol(order, 0, 0, kind=0))   # paper adaptive
+        out.append(pol(order, 0, 0, kind=1))   # tuned adaptive
+    return out
+
+
+def pname(p):
+    return f"{'O' if p.order else 'U'}_{'auto' if not p.mapping else A.MAP_LETTER[p.mapping]}_" \
+           f"{'auto' if not p.workset else A.WS_NAME[p.workset]}_{'paper' if p.kind == 0 else 'tuned'}"
+
+
+def check_bfs(g, G, s, p, expect_level=None):
+    lv, par = oracle.bfs(g, s) if expect_level is None else (expect_level, None)
+    parents = np.empty(g.V, np.uint32)
+    out, _, st = G.bfs(s, parents=parents, policy=p, stats=True, trace_cap=1 << 16)
+    assert np.array_equal(out, lv), f"BFS levels differ ({pname(p)}, src {s}): " \
+        f"{np.count_nonzero(out != lv)} mismatches"
+    code, bad = oracle.validate(g, s, out, parents, weighted=False)
+    assert code == 0, f"BFS parent certificate failed: {oracle.VALIDATE_MSG[code]} at {bad} ({pname(p)})"
+    Vr, Er = oracle.reached(g, lv)
+    assert (st.reached, st.reached_edges) == (Vr, Er)
+    # level-synchronous: ordered AND unordered BFS expand each reached vertex exactly once (16.s43, 26.s33)
+    assert st.vertices_expanded == Vr and st.edges_inspected == Er
+    assert st.iterations == oracle.bfs_iterations(lv)
+    assert list(st.trace_ws) == list(oracle.bfs_level_sizes(lv))
+    assert list(st.trace_edges) == list(oracle.bfs_level_edges(g, lv))
+    return st
+
+
+def check_sssp(g, G, s, p):
+    d, _ = oracle.dijkstra(g, s)
+    parents = np.empty(g.V, np.uint32)
+    out, _, st = G.sssp(s, parents=parents, policy=p, stats=True)
+    assert np.array_equal(out, d), f"SSSP dist differ ({pname(p)}, src {s}): {np.count_nonzero(out != d)} mismatches"
+    code, bad = oracle.validate(g, s, out, parents, weighted=True)
+    assert code == 0, f"SSSP parent certificate failed: {oracle.VALIDATE_MSG[code]} at {bad} ({pname(p)})"
+    Vr, Er = oracle.reached(g, d)
+    assert (st.reached, st.reached_edges) == (Vr, Er)
+    if p.order == 1 and p.delta == 1:
+        # Dijkstra batches: each vertex settled exactly once (18.s2); one iteration per distinct distance (28.s8)
+        assert st.vertices_expanded == Vr and st.edges_inspected == Er
+        assert st.iterations == oracle.ordered_sssp_iterations(d)
+    else:
+        assert st.vertices_expanded >= Vr and st.edges_inspected >= Er
+    return st
+
+
+# ------------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("seed", range(8))
+def test_tiny_random_all_variants(seed):
+    rng = np.random.default_rng(seed)
+    V = int(rng.integers(1, 300))
+    g = aggen.random_graph(V, int(rng.integers(0, 6 * V + 1)), seed=seed, wmax=int(rng.integers(1, 100)),
+                           sort_rows=bool(seed % 2))
+    G = A.Graph.from_csr(g)
+    srcs = sorted(set([0, V - 1, int(rng.integers(0, V))]))
+    for p in all_policies():
+        for s in srcs:
+            check_bfs(g, G, s, p)
+            check_sssp(g, G, s, p)
+
+
+@pytest.mark.parametrize("delta", [1, 7, 100, 1000])
+def test_ordered_sssp_delta(delta):
+    g = aggen.config("C1")
+    G = A.Graph.from_csr(g)
+    for s in aggen.sources(g, 3):
+        for w in WSS:
+            check_sssp(g, G, s, pol(1, 4, w, delta=delta))
+            check_sssp(g, G, s, pol(1, 1, w, delta=delta))
+
+
+def test_c1_all_sources_adaptive():
+    """C1 (R-MAT s12 ef16): all 64 sources, BFS + SSSP, adaptive tuned and paper policies."""
+    g = aggen.config("C1")
+    G = A.Graph.from_csr(g)
+    for s in aggen.sources(g, 64):
+        for kind in (0, 1):
+            check_bfs(g, G, s, pol(0, kind=kind))
+            check_sssp(g, G, s, pol(0, kind=kind))
+
+
+def test_c1_all_static_variants():
+    g = aggen.config("C1")
+    G = A.Graph.from_csr(g)
+    for s in aggen.sources(g, 4, seed=11):
+        for p in all_policies():
+            check_bfs(g, G, s, p)
+            check_sssp(g, G, s, p)
+
+
+def test_paper_policy_trace_matches_fig11():
+    """The per-iteration variant chosen on device == Fig. 11 applied to the oracle's level sizes."""
+    g = aggen.rmat(16, 16, seed=1)
+    G = A.Graph.from_csr(g, weighted=False)
+    p = pol(0, kind=0)
+    T3 = selector.t3_from_ppm(g.V, p.t3_ppm)
+    for s in aggen.sources(g, 3):
+        st = check_bfs(g, G, s, p)
+        lv, _ = oracle.bfs(g, s)
+        exp = [selector.paper_select(int(n), g.V, g.E, T1=p.t1_avg_degree, T2=p.t2_ws, T3=T3)
+               for n in oracle.bfs_level_sizes(lv)]
+        got = [tuple(A.variant_name(int(v)).split("_")) for v in st.trace_variant]
+        assert got == exp
+
+
+def test_closed_form_grid_and_path():
+    W, H = 300, 200
+    g = aggen.grid(W, H)
+    g.w = aggen.weights(g, seed=3, wmax=0)
+    G = A.Graph.from_csr(g)
+    y, x = np.divmod(np.arange(W * H), W)
+    for sx, sy in [(0, 0), (299, 199), (123, 45)]:
+        man = (np.abs(x - sx) + np.abs(y - sy)).astype(np.uint32)
+        for p in (pol(0), pol(1), pol(0, 1, 2), pol(0, 1, 1)):
+            out, _, _ = G.bfs(sy * W + sx, policy=p)
+            assert np.array_equal(out, man)
+            out, _, _ = G.sssp(sy * W + sx, policy=p)
+            assert np.array_equal(out, 3 * man)
+    g = aggen.path(5000)
+    G = A.Graph.from_csr(g, weighted=False)
+    out, _, st = G.bfs(17, policy=pol(0), stats=True)
+    assert np.array_equal(out, np.abs(np.arange(5000) - 17).astype(np.uint32)) and st.iterations == 4983
+
+
+def test_hubs_and_star():
+    """Degree >> HUB_DEG exercises hub splitting (hybrid) and long CTA loops (paper variants)."""
+    n = 300_000
+    g = aggen.star(n)
+    aggen.with_weights(g, seed=4, wmax=100)
+    G = A.Graph.from_csr(g)
+    for p in [pol(0), pol(1), pol(0, 4, 2), pol(0, 4, 1), pol(0, 1, 2), pol(0, 3, 1), pol(1, 4, 2)]:
+        for s in (0, 5):
+            check_bfs(g, G, s, p)
+            check_sssp(g, G, s, p)
+
+
+def test_edge_cases_and_errors():
+    g1 = aggen.csr_from_edges(1, [], [], w=[])
+    G = A.Graph.from_csr(g1)
+    out, _, st = G.bfs(0, stats=True)
+    assert list(out) == [0] and st.iterations == 1
+    out, par, _ = G.sssp(0, parents=np.empty(1, np.uint32))
+    assert list(out) == [0] and list(par) == [0]
+    with pytest.raises(A.AgError) as e:
+        G.bfs(1)
+    assert e.value.status == "AG_ERR_SRC_RANGE"
+    # isolated source
+    g = aggen.csr_from_edges(5, [1, 2], [2, 3], w=[1, 1])
+    G = A.Graph.from_csr(g)
+    out, par, _ = G.bfs(0, parents=np.empty(5, np.uint32))
+    assert list(out) == [0, INF, INF, INF, INF] and list(par) == [0, INF, INF, INF, INF]
+    # SSSP without weights
+    Gu = A.Graph.from_csr(g, weighted=False)
+    with pytest.raises(A.AgError) as e:
+        Gu.sssp(0)
+    assert e.value.status == "AG_ERR_NO_WEIGHTS"
+    # bad CSR
+    for rp, col, w in [([1, 1, 2], [0, 1], None), ([0, 2, 1], [0, 1], None), ([0, 1, 2], [0, 5], None),
+                       ([0, 1, 2], [0, 1], [1, 0]), ([0, 1, 2], [0, 1], [1, 1 << 31])]:
+        with pytest.raises(A.AgError) as e:
+            A.Graph(2, np.array(rp, np.uint64), np.array(col, np.uint32), None if w is None else np.array(w, np.uint32))
+        assert e.value.status == "AG_ERR_BAD_CSR"
+    # overflow: path with huge weights
+    g = aggen.path(4)
+    g.w = np.full(g.E, 0x7FFFFFFF, np.uint32)
+    G = A.Graph.from_csr(g)
+    for order in (0, 1):
+        with pytest.raises(A.AgError) as e:
+            G.sssp(0, policy=pol(order))
+        assert e.value.status == "AG_ERR_OVERFLOW"
+    g3 = aggen.path(3)
+    g3.w = np.full(g3.E, 0x7FFFFFFF, np.uint32)
+    out, _, _ = A.Graph.from_csr(g3).sssp(0)
+    assert list(out) == [0, 0x7FFFFFFF, 0xFFFFFFFE]
+
+
+def test_device_buffers_and_async():
+    import torch
+    g = aggen.config("C1")
+    G = A.Graph.from_csr(g)
+    s = int(aggen.sources(g, 1)[0])
+    lv, _ = oracle.bfs(g, s)
+    d, _ = oracle.dijkstra(g, s)
+    out = torch.empty(g.V, dtype=torch.int32, device="cuda")
+    par = torch.empty(g.V, dtype=torch.int32, device="cuda")
+    stream = torch.cuda.current_stream().cuda_stream
+    G.bfs(s, levels=out, parents=par, stream=stream)        # enqueued only
+    G.check()
+    assert np.array_equal(out.cpu().numpy().view(np.uint32), lv)
+    assert oracle.validate(g, s, out.cpu().numpy().view(np.uint32), par.cpu().numpy().view(np.uint32))[0] == 0
+    G.sssp(s, dist=out, parents=par, stream=stream)
+    G.check()
+    assert np.array_equal(out.cpu().numpy().view(np.uint32), d)
+    # device-resident CSR input
+    t_rp = torch.from_numpy(g.row_ptr.view(np.int64)).cuda()
+    t_col = torch.from_numpy(g.col.view(np.int32)).cuda()
+    t_w = torch.from_numpy(g.w.view(np.int32)).cuda()
+    G2 = A.Graph(g.V, t_rp, t_col, t_w)
+    out2, _, _ = G2.sssp(s)
+    assert np.array_equal(out2, d)
+
+
+# ------------------------------------------------------------------------------------------------
+# full-size configs (BASELINE.json), in the launch configuration bench.py times
+# ------------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("cfg", ["C2", "C3", "C3p", "C4"])
+def test_full_size_configs(cfg):
+    g = aggen.config(cfg)
+    G = A.Graph.from_csr(g)
+    srcs = [0] if cfg.startswith("C3") else []
+    srcs += [int(s) for s in aggen.sources(g, 2)]
+    for s in srcs:
+        check_bfs(g, G, s, pol(0))
+        check_sssp(g, G, s, pol(0))
+        if cfg == "C2":
+            check_bfs(g, G, s, pol(0, kind=0))
+            check_bfs(g, G, s, pol(1))
+    if cfg in ("C3", "C3p"):
+        check_sssp(g, G, srcs[-1], pol(1, delta=1 if cfg == "C3p" else 64))
