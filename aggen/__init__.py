@@ -230,6 +230,8 @@ def config(name: str, weighted: bool = True) -> Graph:
         g = rmat(26, 16, seed=1)
     elif name.startswith("rmat"):
         g = rmat(int(name[4:]), 16, seed=1)
+    elif name.startswith("path"):     # per-iteration latency floor (one vertex per level)
+        g = path(int(name[4:]))
     else:
         raise KeyError(name)
     g.name = name

@@ -1,0 +1,342 @@
+#!/usr/bin/env python
+"""bench.py — BFS/SSSP GTEPS on B200, device-timed, with the HBM-roofline fraction.
+
+One STEP = one pass of the whole hot path over one query of the workload: an adaptive BFS and an
+adaptive (unordered) SSSP from source s_k of config C2 (R-MAT scale 22, edgefactor 16, weights
+1..100; BASELINE.json configs[1]).  value = (E_r(BFS) + E_r(SSSP)) / time, in GTEPS
+(E_r = CSR entries whose source is reached, R20).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl agraph|reference] [--config C2]
+
+N > 1 (torchrun): every rank runs independent queries (different sources) on its own GPU —
+independent problems, no data-path collective — "scaling": "weak".
+--impl reference: the CPU oracle (serial queue BFS + heap Dijkstra, the paper's own baselines,
+PAPER.md:26.s21, 26.s36) timed on this host, rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+CONFIG_DESC = {
+    "C1": "R-MAT scale-12 ef16, weights 1..100",
+    "C2": "R-MAT scale-22 ef16, weights 1..100",
+    "C3": "2-D grid 4096x4096 (road-like, diameter 8190), weights 1..100",
+    "C3p": "2-D grid 4096x4096 bond-percolated keep 0.6 (CO-road avg deg 2.4), weights 1..100",
+    "C4": "Erdos-Renyi n=2^25 m=4n (avg deg 8), weights 1..100",
+}
+
+
+def env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+def measured_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons with NVML while the timed region runs."""
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, device):
+        self.samples, self.reasons, self.ok = [], 0, False
+        self.max_mhz = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            pass
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                self.reasons |= int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+            except Exception:
+                pass
+            time.sleep(0.002)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.ok:
+            self.t.join()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["unavailable"]}
+        names = [n for b, n in self.REASONS.items() if self.reasons & b and n != "gpu_idle"]
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz, "reasons": names,
+                "samples": len(self.samples)}
+
+
+def algorithmic_bytes(V, Vr, Er, off_bytes, sssp):
+    """Compulsory bytes of one traversal: init out[] 4V, row-offset pair + result
+    write per reached vertex, col_idx per reached edge (+ weight per reached edge for SSSP)."""
+    b = 4 * V + (2 * off_bytes + 4) * Vr + 4 * Er
+    if sssp:
+        b += 4 * Er
+    return b
+
+
+def load_traffic(cfg):
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        return json.load(open(p)).get(cfg)
+    except Exception:
+        return None
+
+
+def run_reference(args, rank, world):
+    """The oracle as it stands, on this host's cores (rank 0 only)."""
+    if rank != 0:
+        return
+    import aggen
+    import oracle
+    g = aggen.config(args.config)
+    srcs = aggen.sources(g, 64, seed=3)
+    budget_s = float(os.environ.get("AG_REF_BUDGET_S", "150"))
+    t_step, edges, ran = [], [], 0
+    t0 = time.time()
+    total = args.warmup + args.steps
+    for k in range(total):
+        s = int(srcs[k % len(srcs)])
+        ts = time.perf_counter()
+        lv, _ = oracle.bfs(g, s, want_parents=False)
+        d, _ = oracle.dijkstra(g, s, want_parents=False)
+        dt = time.perf_counter() - ts
+        if k >= args.warmup or (ran == 0 and time.time() - t0 > budget_s / 2):
+            _, e1 = oracle.reached(g, lv)
+            _, e2 = oracle.reached(g, d)
+            t_step.append(dt)
+            edges.append(e1 + e2)
+            ran += 1
+        if time.time() - t0 > budget_s and ran >= 1:
+            break
+    tot_t, tot_e = sum(t_step), sum(edges)
+    val = tot_e / tot_t / 1e9
+    sample = f"{ran} of {args.steps} steps (1 BFS + 1 Dijkstra from one source each) on {args.config}, " \
+             f"budget {budget_s:.0f}s"
+    out = {"metric": "BFS/SSSP GTEPS (device-timed); fraction of HBM roofline", "impl": "reference",
+           "value": val, "unit": "GTEPS", "n_gpus": world, "steps": ran, "warmup": args.warmup,
+           "ms_per_step": 1e3 * tot_t / ran, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+           "dtype": "u32", "data": "synthetic",
+           "config": {"workload": f"{args.config}: {CONFIG_DESC.get(args.config, '')}; BFS + SSSP per step",
+                      "V": g.V, "E": g.E},
+           "cpu_baseline": {"value": val, "unit": "GTEPS", "cores": 1, "kind": "oracle", "sample": sample},
+           "e2e": {"value": val, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def cpu_baseline(g, srcs, budget_s=20.0):
+    import oracle
+    t, e, n = 0.0, 0, 0
+    for s in srcs:
+        ts = time.perf_counter()
+        lv, _ = oracle.bfs(g, int(s), want_parents=False)
+        d, _ = oracle.dijkstra(g, int(s), want_parents=False)
+        t += time.perf_counter() - ts
+        e += oracle.reached(g, lv)[1] + oracle.reached(g, d)[1]
+        n += 1
+        if t > budget_s:
+            break
+    return {"value": e / t / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+            "sample": f"{n} sources x (queue BFS + heap Dijkstra) on the full graph, serial, {t:.1f}s"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="agraph", choices=["agraph", "reference"])
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    world = env_int("WORLD_SIZE", 1)
+    rank = env_int("RANK", 0)
+    local = env_int("LOCAL_RANK", 0)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import aggen
+    from paper_conf_ipps_lib13_b200 import agraph as A
+    from paper_conf_ipps_lib13_b200 import build as B
+
+    B.build()
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    g = aggen.config(args.config)
+    G = A.Graph.from_csr(g, device=local)
+    srcs = aggen.sources(g, 64, seed=3)
+    pol = A.policy_default(local)
+    stream = torch.cuda.current_stream()
+    sp = stream.cuda_stream
+    V = g.V
+    lev = torch.empty(V, dtype=torch.int32, device="cuda")
+    dist_out = torch.empty(V, dtype=torch.int32, device="cuda")
+
+    # per-source reached counts (E_r, V_r) — measured once, outside the timed region
+    info = {}
+    for s in sorted(set(int(x) for x in srcs)):
+        _, _, sb = G.bfs(s, levels=lev, policy=pol, stats=True)
+        _, _, ss = G.sssp(s, dist=dist_out, policy=pol, stats=True)
+        info[s] = (sb.reached, sb.reached_edges, ss.reached, ss.reached_edges, sb.iterations, ss.iterations,
+                   ss.edges_inspected)
+
+    def step_src(k):
+        return int(srcs[(k * world + rank) % len(srcs)])
+
+    for k in range(args.warmup):
+        s = step_src(k)
+        G.bfs(s, levels=lev, policy=pol, stream=sp)
+        G.sssp(s, dist=dist_out, policy=pol, stream=sp)
+    torch.cuda.synchronize()
+
+    K = args.steps
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(K)]
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    launches0 = A.kernel_launches()
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize()
+    sampler = ClockSampler(local)
+    with sampler:
+        start.record(stream)
+        for k in range(K):
+            s = step_src(k)
+            ev[k][0].record(stream)
+            G.bfs(s, levels=lev, policy=pol, stream=sp)
+            ev[k][1].record(stream)
+            G.sssp(s, dist=dist_out, policy=pol, stream=sp)
+            ev[k][2].record(stream)
+        end.record(stream)
+        torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    G.check()
+    launches = A.kernel_launches() - launches0
+    t_ms = start.elapsed_time(end)
+    t_bfs = [ev[k][0].elapsed_time(ev[k][1]) for k in range(K)]
+    t_sssp = [ev[k][1].elapsed_time(ev[k][2]) for k in range(K)]
+    e_bfs = sum(info[step_src(k)][1] for k in range(K))
+    e_sssp = sum(info[step_src(k)][3] for k in range(K))
+    edges = e_bfs + e_sssp
+    if dist:
+        tt = torch.tensor([t_ms], device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_ms = float(tt.item())
+        ee = torch.tensor([edges], dtype=torch.float64, device="cuda")
+        dist.all_reduce(ee)
+        edges = float(ee.item())
+    value = edges / (t_ms * 1e-3) / 1e9
+
+    # roofline of the dominant kernel (the traversal kernel that takes more of the step)
+    peak, peak_src = measured_peak()
+    off = G.info.offset_bytes
+    b_bfs = sum(algorithmic_bytes(V, info[step_src(k)][0], info[step_src(k)][1], off, False) for k in range(K)) / K
+    b_sssp = sum(algorithmic_bytes(V, info[step_src(k)][2], info[step_src(k)][3], off, True) for k in range(K)) / K
+    mb, ms_ = statistics.mean(t_bfs), statistics.mean(t_sssp)
+    if ms_ >= mb:
+        dom, db, dt = "sssp", b_sssp, ms_
+    else:
+        dom, db, dt = "bfs", b_bfs, mb
+    achieved = db / (dt * 1e-3) / 1e9
+    traffic = load_traffic(f"{args.config}:{dom}")
+    roof = {"bound": "hbm", "kernel": f"traverse_kernel ({dom})", "achieved": achieved, "peak": peak,
+            "peak_source": peak_src, "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+            "algorithmic_bytes_per_launch": db,
+            "bfs": {"ms": mb, "GBps": b_bfs / (mb * 1e-3) / 1e9, "frac": b_bfs / (mb * 1e-3) / 1e9 / peak},
+            "sssp": {"ms": ms_, "GBps": b_sssp / (ms_ * 1e-3) / 1e9, "frac": b_sssp / (ms_ * 1e-3) / 1e9 / peak}}
+
+    out = {"metric": "BFS/SSSP GTEPS (device-timed); fraction of HBM roofline", "value": value, "unit": "GTEPS",
+           "n_gpus": world, "steps": K, "warmup": args.warmup, "ms_per_step": t_ms / K, "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+           "config": {"workload": f"{args.config}: {CONFIG_DESC.get(args.config, '')}; one step = adaptive BFS + "
+                                  f"adaptive unordered SSSP from one of 64 seeded sources",
+                      "V": V, "E": g.E, "sources": len(srcs), "policy": "tuned adaptive (ag_policy_default)",
+                      "l2": "inputs larger than L2 (CSR col+w = %.2f GB > 126 MB)" % (g.E * 8 / 1e9),
+                      "parallelism": f"{world} independent replica(s)" if world > 1 else "1 GPU"},
+           "bfs_gteps": e_bfs / (sum(t_bfs) * 1e-3) / 1e9, "sssp_gteps": e_sssp / (sum(t_sssp) * 1e-3) / 1e9,
+           "iterations": {"bfs": statistics.mean(info[step_src(k)][4] for k in range(K)),
+                          "sssp": statistics.mean(info[step_src(k)][5] for k in range(K))},
+           "sssp_redundancy": statistics.mean(info[step_src(k)][6] / max(1, info[step_src(k)][3]) for k in range(K)),
+           "roofline": roof, "gpu_launches": launches, "clocks": sampler.summary()}
+
+    # end-to-end through the public API with HOST buffers: CSR upload from pinned memory, both
+    # traversals, results read back (the paper's timing scope, 26.s17-18; reading R21)
+    if not args.no_e2e:
+        rp_h = torch.from_numpy(g.row_ptr.view(np.int64)).pin_memory()
+        col_h = torch.from_numpy(g.col.view(np.int32)).pin_memory()
+        w_h = torch.from_numpy(g.w.view(np.int32)).pin_memory()
+        lv_h = torch.empty(V, dtype=torch.int32).pin_memory()
+        d_h = torch.empty(V, dtype=torch.int32).pin_memory()
+        ke = min(K, 5)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        e2e_edges = 0
+        for k in range(ke):
+            s = step_src(k)
+            Gh = A.Graph(V, rp_h, col_h, w_h, device=local)
+            Gh.bfs(s, levels=lv_h, policy=pol, stream=sp)
+            Gh.sssp(s, dist=d_h, policy=pol, stream=sp)
+            Gh.free()
+            e2e_edges += info[s][1] + info[s][3]
+        torch.cuda.synchronize()
+        t_e2e = time.perf_counter() - t0
+        h2d = g.row_ptr.nbytes + g.col.nbytes + g.w.nbytes
+        out["e2e"] = {"value": e2e_edges / t_e2e / 1e9, "unit": "GTEPS", "h2d_bytes_per_step": int(h2d),
+                      "d2h_bytes_per_step": int(2 * 4 * V), "steps": ke,
+                      "scope": "ag_graph_load_csr(pinned host CSR) + ag_bfs + ag_sssp (host outputs) + ag_graph_free"}
+
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        out["cpu_baseline"] = cpu_baseline(g, [step_src(k) for k in range(3)],
+                                           budget_s=float(os.environ.get("AG_CPU_BUDGET_S", "20")))
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -99,8 +99,15 @@ typedef struct {
     int32_t device;              /* CUDA device ordinal */
     uint32_t num_sms;            /* SM count of that device */
     uint32_t offset_bytes;       /* 4 if row offsets are stored as u32 (E < 2^32), else 8 */
-    uint32_t reserved;
+    uint32_t layout;             /* ag_layout actually used (IDENTITY or DEGREE) */
 } ag_graph_info;
+
+/* Device vertex layout.  DEGREE relabels vertices by descending out-degree at load
+ * time so that the status words of high-degree vertices — the targets of most edges in a power-law
+ * graph — are packed into a small, cache-resident prefix of the visited bitmap / state arrays.
+ * Results are always returned in the caller's vertex ids.  AUTO picks DEGREE when the inspector
+ * sees a skewed degree distribution (max_deg >= 64 x ceil(E/V)), else IDENTITY. */
+typedef enum { AG_LAYOUT_AUTO = 0, AG_LAYOUT_IDENTITY = 1, AG_LAYOUT_DEGREE = 2 } ag_layout;
 
 typedef struct {
     uint32_t struct_size;        /* caller sets sizeof(ag_run_stats) */
@@ -116,6 +123,9 @@ typedef struct {
     uint32_t *trace_ws;          /* per iteration |WS| (host, nullable) */
     uint64_t *trace_edges;       /* per iteration edges inspected (host, nullable) */
     uint8_t *trace_variant;      /* per iteration variant id AG_VARIANT(m, w) (host, nullable) */
+    uint64_t *trace_ns;          /* per iteration device timestamp (ns, %globaltimer) at the start
+                                    of the iteration; entry [iterations] = end (host, nullable,
+                                    capacity trace_cap + 1) */
 } ag_run_stats;
 
 /* ---------------------------------------------------------------------------------------------
@@ -143,6 +153,9 @@ uint8_t ag_select(const ag_policy *p, const ag_graph_info *gi, uint64_t ws_size,
  * *out receives the handle (owned by the library until ag_graph_free). */
 ag_status ag_graph_load_csr(uint32_t V, uint64_t E, const uint64_t *row_ptr, const uint32_t *col_idx,
                             const uint32_t *weights, int device, ag_graph *out);
+/* As ag_graph_load_csr with an explicit device layout (ag_layout). */
+ag_status ag_graph_load_csr_ex(uint32_t V, uint64_t E, const uint64_t *row_ptr, const uint32_t *col_idx,
+                               const uint32_t *weights, int device, uint32_t layout, ag_graph *out);
 ag_status ag_graph_info_get(ag_graph g, ag_graph_info *out);
 ag_status ag_graph_free(ag_graph g);
 

@@ -14,7 +14,7 @@ from typing import Optional
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libagraph.so")
+LIB_PATH = os.environ.get("AGRAPH_LIB") or os.path.join(HERE, "libagraph.so")  # override: experiment builds
 INF = 0xFFFFFFFF
 
 # enums (include/agraph.h)
@@ -22,6 +22,7 @@ UNORDERED, ORDERED = 0, 1
 MAP_AUTO, MAP_THREAD, MAP_WARP, MAP_CTA, MAP_HYBRID = 0, 1, 2, 3, 4
 WS_AUTO, WS_BITMAP, WS_QUEUE = 0, 1, 2
 POLICY_PAPER, POLICY_TUNED = 0, 1
+LAYOUT_AUTO, LAYOUT_IDENTITY, LAYOUT_DEGREE = 0, 1, 2
 STATUS = {0: "AG_OK", 1: "AG_ERR_INVALID_ARG", 2: "AG_ERR_BAD_CSR", 3: "AG_ERR_SRC_RANGE", 4: "AG_ERR_NO_WEIGHTS",
           5: "AG_ERR_OVERFLOW", 6: "AG_ERR_OOM", 7: "AG_ERR_CUDA", 8: "AG_ERR_NCCL", 9: "AG_ERR_UNSUPPORTED",
           10: "AG_ERR_NO_DEVICE"}
@@ -56,7 +57,7 @@ class GraphInfo(ctypes.Structure):
     _fields_ = [("num_vertices", ctypes.c_uint32), ("min_deg", ctypes.c_uint32), ("max_deg", ctypes.c_uint32),
                 ("num_edges", ctypes.c_uint64), ("deg_sum", ctypes.c_uint64), ("isolated", ctypes.c_uint32),
                 ("weighted", ctypes.c_uint32), ("device", ctypes.c_int32), ("num_sms", ctypes.c_uint32),
-                ("offset_bytes", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
+                ("offset_bytes", ctypes.c_uint32), ("layout", ctypes.c_uint32)]
 
 
 class RunStats(ctypes.Structure):
@@ -65,10 +66,10 @@ class RunStats(ctypes.Structure):
                 ("reached", ctypes.c_uint64), ("reached_edges", ctypes.c_uint64), ("device_ms", ctypes.c_float),
                 ("trace_cap", ctypes.c_uint32), ("trace_len", ctypes.c_uint32), ("reserved", ctypes.c_uint32),
                 ("trace_ws", ctypes.POINTER(ctypes.c_uint32)), ("trace_edges", ctypes.POINTER(ctypes.c_uint64)),
-                ("trace_variant", ctypes.POINTER(ctypes.c_uint8))]
+                ("trace_variant", ctypes.POINTER(ctypes.c_uint8)), ("trace_ns", ctypes.POINTER(ctypes.c_uint64))]
 
 
-EXPORTS = ["ag_policy_default", "ag_select", "ag_graph_load_csr", "ag_graph_info_get", "ag_graph_free", "ag_bfs",
+EXPORTS = ["ag_policy_default", "ag_select", "ag_graph_load_csr", "ag_graph_load_csr_ex", "ag_graph_info_get", "ag_graph_free", "ag_bfs",
            "ag_sssp", "ag_graph_check", "ag_dist_unique_id", "ag_dist_init", "ag_dist_free", "ag_dist_owned_range",
            "ag_dist_graph_load_csr", "ag_dist_bfs", "ag_set_allocator", "ag_status_string", "ag_last_error",
            "ag_abi_version", "ag_kernel_launches"]
@@ -89,6 +90,7 @@ def lib():
     L.ag_select.argtypes = [ctypes.POINTER(Policy), ctypes.POINTER(GraphInfo), u64, u64]
     L.ag_select.restype = ctypes.c_uint8
     L.ag_graph_load_csr.argtypes = [u32, u64, vp, vp, vp, i32, ctypes.POINTER(vp)]
+    L.ag_graph_load_csr_ex.argtypes = [u32, u64, vp, vp, vp, i32, u32, ctypes.POINTER(vp)]
     L.ag_graph_info_get.argtypes = [vp, ctypes.POINTER(GraphInfo)]
     L.ag_graph_free.argtypes = [vp]
     L.ag_graph_check.argtypes = [vp]
@@ -154,23 +156,24 @@ class Stats:
     trace_ws: np.ndarray = field(default_factory=lambda: np.zeros(0, np.uint32))
     trace_edges: np.ndarray = field(default_factory=lambda: np.zeros(0, np.uint64))
     trace_variant: np.ndarray = field(default_factory=lambda: np.zeros(0, np.uint8))
+    trace_us: np.ndarray = field(default_factory=lambda: np.zeros(0, np.float64))  # per-iteration device time
 
 
 class Graph:
     """A graph loaded into device memory (ag_graph_load_csr)."""
 
-    def __init__(self, V: int, row_ptr, col, w=None, device: int = 0):
+    def __init__(self, V: int, row_ptr, col, w=None, device: int = 0, layout: int = LAYOUT_AUTO):
         h = ctypes.c_void_p()
         E = int(row_ptr[-1]) if isinstance(row_ptr, np.ndarray) else int(row_ptr[-1].item())
-        _check(lib().ag_graph_load_csr(V, E, _ptr(row_ptr), _ptr(col), _ptr(w), device, ctypes.byref(h)))
+        _check(lib().ag_graph_load_csr_ex(V, E, _ptr(row_ptr), _ptr(col), _ptr(w), device, layout, ctypes.byref(h)))
         self.h = h
         self.V, self.E, self.device = V, E, device
         self.info = GraphInfo()
         _check(lib().ag_graph_info_get(self.h, ctypes.byref(self.info)))
 
     @classmethod
-    def from_csr(cls, g, device: int = 0, weighted: bool = True):
-        return cls(g.V, g.row_ptr, g.col, g.w if weighted else None, device)
+    def from_csr(cls, g, device: int = 0, weighted: bool = True, layout: int = LAYOUT_AUTO):
+        return cls(g.V, g.row_ptr, g.col, g.w if weighted else None, device, layout)
 
     def free(self):
         if self.h:
@@ -192,11 +195,13 @@ class Graph:
             st = RunStats()
             st.struct_size = ctypes.sizeof(RunStats)
             if trace_cap:
-                tr = (np.zeros(trace_cap, np.uint32), np.zeros(trace_cap, np.uint64), np.zeros(trace_cap, np.uint8))
+                tr = (np.zeros(trace_cap, np.uint32), np.zeros(trace_cap, np.uint64), np.zeros(trace_cap, np.uint8),
+                      np.zeros(trace_cap + 1, np.uint64))
                 st.trace_cap = trace_cap
                 st.trace_ws = tr[0].ctypes.data_as(ctypes.POINTER(ctypes.c_uint32))
                 st.trace_edges = tr[1].ctypes.data_as(ctypes.POINTER(ctypes.c_uint64))
                 st.trace_variant = tr[2].ctypes.data_as(ctypes.POINTER(ctypes.c_uint8))
+                st.trace_ns = tr[3].ctypes.data_as(ctypes.POINTER(ctypes.c_uint64))
         rc = fn(self.h, int(src), _ptr(out), _ptr(parents), ctypes.byref(policy) if policy is not None else None,
                 ctypes.byref(st) if st is not None else None, ctypes.c_void_p(stream or 0))
         _check(rc)
@@ -207,6 +212,8 @@ class Graph:
                         st.device_ms)
             if tr is not None:
                 res.trace_ws, res.trace_edges, res.trace_variant = tr[0][:n], tr[1][:n], tr[2][:n]
+                if n == st.iterations:
+                    res.trace_us = np.diff(tr[3][:n + 1].astype(np.float64)) / 1e3
         return out, parents, res
 
     def bfs(self, src: int, levels=None, parents=None, policy: Optional[Policy] = None, stats: bool = False,

@@ -5,6 +5,7 @@
 #include <atomic>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -142,6 +143,11 @@ __global__ void validate_edges_kernel(const uint32_t *col, const uint32_t *w, ui
     if ((threadIdx.x & 31) == 0 && bad) atomicOr(&st->bad, bad);
 }
 
+__global__ void interleave_kernel(const uint32_t *col, const uint32_t *w, uint2 *cw, uint64_t E) {
+    for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < E; e += (uint64_t)gridDim.x * blockDim.x)
+        cw[e] = make_uint2(col[e], w[e]);
+}
+
 __global__ void narrow_offsets_kernel(const uint64_t *rp, uint32_t *rp32, uint32_t n) {
     for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
         rp32[i] = (uint32_t)rp[i];
@@ -149,10 +155,15 @@ __global__ void narrow_offsets_kernel(const uint64_t *rp, uint32_t *rp32, uint32
 
 // V_r and E_r of a result array (stats only; not in the timed path)
 template <typename Off>
-__global__ void reached_kernel(const uint32_t *out, const Off *rp, uint32_t V, unsigned long long *acc) {
+__global__ void reached_kernel(const uint32_t *out, const Off *rp, const uint32_t *inv, uint32_t V,
+                               unsigned long long *acc) {
     unsigned long long a = 0, b = 0;
     for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x)
-        if (out[v] != INF) { a += 1; b += (unsigned long long)(rp[v + 1] - rp[v]); }
+        if (out[v] != INF) {
+            const uint32_t i = inv ? inv[v] : v;
+            a += 1;
+            b += (unsigned long long)(rp[i + 1] - rp[i]);
+        }
     a = warp_sum(a);
     b = warp_sum(b);
     if ((threadIdx.x & 31) == 0 && (a | b)) { atomicAdd(&acc[0], a); atomicAdd(&acc[1], b); }
@@ -160,12 +171,15 @@ __global__ void reached_kernel(const uint32_t *out, const Off *rp, uint32_t V, u
 
 // exact overflow test after a flagged SSSP: a reachable vertex left at INF behind a finite one
 template <typename Off>
-__global__ void overflow_check_kernel(const uint32_t *dist, const Off *rp, const uint32_t *col, uint32_t V,
-                                      unsigned *flag) {
+__global__ void overflow_check_kernel(const uint32_t *dist, const Off *rp, const uint32_t *col, const uint32_t *perm,
+                                      uint32_t V, unsigned *flag) {
+    // rp/col in device-layout ids, dist in caller ids
     for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < V; u += gridDim.x * blockDim.x) {
-        if (dist[u] == INF) continue;
-        for (Off e = rp[u]; e < rp[u + 1]; ++e)
-            if (dist[col[e]] == INF) { *flag = 1; return; }
+        if (dist[perm ? perm[u] : u] == INF) continue;
+        for (Off e = rp[u]; e < rp[u + 1]; ++e) {
+            const uint32_t v = col[e];
+            if (dist[perm ? perm[v] : v] == INF) { *flag = 1; return; }
+        }
     }
 }
 
@@ -229,6 +243,8 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
     d.cta_group = grp;
     d.V = g.V;
     d.E = g.E;
+    d.max_deg = g.info.max_deg;
+    d.t2_tuned = 65536;
     return d;
 }
 
@@ -253,8 +269,34 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, BS, 0);
     if (e != cudaSuccess || occ < 1) return cuda_status(e == cudaSuccess ? cudaErrorLaunchOutOfResources : e, "occupancy");
     a.nblocks = (uint32_t)(occ * g->num_sms);
-    void *args[] = {(void *)&a};
-    e = cudaLaunchCooperativeKernel((const void *)fn, dim3(a.nblocks), dim3(BS), args, 0, st);
+    // Cooperative launch (co-resident grid for the software grid barrier) with an L2 access-policy
+    // window marking the per-vertex status array persisting, so the ~1 GB CSR stream does not evict
+    // it.  The window is a per-launch attribute: the caller's stream is not modified.
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(a.nblocks);
+    cfg.blockDim = dim3(BS);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = st;
+    cudaLaunchAttribute attrs[2];
+    attrs[0].id = cudaLaunchAttributeCooperative;
+    attrs[0].val.cooperative = 1;
+    int nattr = 1;
+    void *wbase = ALG == ALG_SSSP ? (void *)a.P : (void *)a.vis;
+    size_t wbytes = ALG == ALG_SSSP ? (size_t)g->V * 8 : (size_t)g->nwords * 4;
+    if (g->persist_bytes > 0 && getenv("AG_NO_L2_WINDOW") == nullptr) {
+        if (wbytes > g->max_window) wbytes = g->max_window;
+        attrs[1].id = cudaLaunchAttributeAccessPolicyWindow;
+        attrs[1].val.accessPolicyWindow.base_ptr = wbase;
+        attrs[1].val.accessPolicyWindow.num_bytes = wbytes;
+        attrs[1].val.accessPolicyWindow.hitRatio =
+            wbytes <= g->persist_bytes ? 1.0f : (float)g->persist_bytes / (float)wbytes;
+        attrs[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        attrs[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        nattr = 2;
+    }
+    cfg.attrs = attrs;
+    cfg.numAttrs = nattr;
+    e = cudaLaunchKernelEx(&cfg, fn, a);
     note_launch(1);
     return cuda_status(e, "traverse launch");
 }
@@ -288,9 +330,10 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
         if ((s = ensure_buf(g, &g->d_par_tmp, &g->par_tmp_bytes, vbytes)) != AG_OK) return s;
         d_par = g->d_par_tmp;
     }
-    uint32_t tcap = (stats && (stats->trace_ws || stats->trace_edges || stats->trace_variant)) ? stats->trace_cap : 0;
+    uint32_t tcap = (stats && (stats->trace_ws || stats->trace_edges || stats->trace_variant || stats->trace_ns))
+                        ? stats->trace_cap : 0;
     if (tcap) {
-        size_t need = (size_t)tcap * 16;
+        size_t need = (size_t)tcap * 24 + 64;
         if ((s = ensure_buf(g, &g->d_trace, &g->trace_bytes, need)) != AG_OK) return s;
     }
 
@@ -298,7 +341,7 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
     memset(&a, 0, sizeof a);
     a.rp = (const Off *)g->d_rp;
     a.col = g->d_col;
-    a.w = g->d_w;
+    a.cw = g->d_cw;
     a.V = g->V;
     a.nwords = g->nwords;
     a.P = g->d_P;
@@ -307,9 +350,21 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
     a.hub = g->d_hub;
     a.hub_cap = g->hub_cap;
     a.ctl = (Ctl *)g->d_ctl;
+    a.perm = g->d_perm;
+    a.inv = g->d_inv;
     if (alg == ALG_BFS) {
-        a.level = d_out;
-        a.parent = d_par;
+        if (g->d_inv) {  // traverse in the degree layout, gather back to caller ids at the end
+            if (!g->d_level && (s = dev_alloc((void **)&g->d_level, (size_t)g->V * 4 + 128, g->device)) != AG_OK) return s;
+            if (d_par && !g->d_lpar && (s = dev_alloc((void **)&g->d_lpar, (size_t)g->V * 4 + 128, g->device)) != AG_OK)
+                return s;
+            a.level = g->d_level;
+            a.parent = d_par ? g->d_lpar : nullptr;
+            a.out_level = d_out;
+            a.out_parent = d_par;
+        } else {
+            a.level = d_out;
+            a.parent = d_par;
+        }
     } else {
         a.dist_out = d_out;
         a.parent_out = d_par;
@@ -319,6 +374,7 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
         a.trace_edges = (unsigned long long *)base;
         a.trace_ws = (uint32_t *)(base + (size_t)tcap * 8);
         a.trace_var = base + (size_t)tcap * 12;
+        a.trace_ns = (unsigned long long *)(base + (((size_t)tcap * 13 + 15) & ~size_t(15)));
         a.trace_cap = tcap;
     }
     a.pol = resolve_policy(pol, *g);
@@ -351,7 +407,7 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
 
     if (stats) {
         cudaMemsetAsync(g->d_acc, 0, 16, st);
-        reached_kernel<Off><<<g->num_sms * 4, 256, 0, st>>>(d_out, (const Off *)g->d_rp, g->V,
+        reached_kernel<Off><<<g->num_sms * 4, 256, 0, st>>>(d_out, (const Off *)g->d_rp, g->d_inv, g->V,
                                                              (unsigned long long *)g->d_acc);
         note_launch(1);
     }
@@ -379,6 +435,9 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
             if (stats->trace_edges) cudaMemcpy(stats->trace_edges, base, (size_t)n * 8, cudaMemcpyDeviceToHost);
             if (stats->trace_ws) cudaMemcpy(stats->trace_ws, base + (size_t)tcap * 8, (size_t)n * 4, cudaMemcpyDeviceToHost);
             if (stats->trace_variant) cudaMemcpy(stats->trace_variant, base + (size_t)tcap * 12, n, cudaMemcpyDeviceToHost);
+            if (stats->trace_ns)
+                cudaMemcpy(stats->trace_ns, base + (((size_t)tcap * 13 + 15) & ~size_t(15)),
+                           (size_t)(c.iterations < tcap ? n + 1 : n) * 8, cudaMemcpyDeviceToHost);
         }
         e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_status(e, "stats");
@@ -448,12 +507,19 @@ uint8_t ag_select(const ag_policy *p, const ag_graph_info *gi, uint64_t ws_size,
     ag_graph_s tmp;
     tmp.V = gi->num_vertices;
     tmp.E = gi->num_edges;
+    tmp.info = *gi;
     DevPolicy d = resolve_policy(*p, tmp);
     return select_variant(d, ws_size, ws_edges);
 }
 
 ag_status ag_graph_load_csr(uint32_t V, uint64_t E, const uint64_t *row_ptr, const uint32_t *col_idx,
                             const uint32_t *weights, int device, ag_graph *out) {
+    return ag_graph_load_csr_ex(V, E, row_ptr, col_idx, weights, device, AG_LAYOUT_AUTO, out);
+}
+
+ag_status ag_graph_load_csr_ex(uint32_t V, uint64_t E, const uint64_t *row_ptr, const uint32_t *col_idx,
+                               const uint32_t *weights, int device, uint32_t layout, ag_graph *out) {
+    if (layout > AG_LAYOUT_DEGREE) return set_error(AG_ERR_INVALID_ARG, "unknown layout %u", layout);
     if (!out || !row_ptr || (!col_idx && E > 0)) return set_error(AG_ERR_INVALID_ARG, "NULL argument");
     *out = nullptr;
     if (V == 0 || V >= 0xFFFFFFFFu) return set_error(AG_ERR_BAD_CSR, "V must be in [1, 2^32-1)");
@@ -503,6 +569,18 @@ ag_status ag_graph_load_csr(uint32_t V, uint64_t E, const uint64_t *row_ptr, con
                               hs.bad & 2 ? "non-monotone row_ptr " : "", hs.bad & 4 ? "row_ptr[V]!=E " : "",
                               hs.bad & 8 ? "col>=V " : "", hs.bad & 16 ? "weight not in [1,2^31) " : ""));
     }
+    // inspector decides the device layout (skewed degree distribution -> degree order)
+    if (layout == AG_LAYOUT_AUTO) {
+        uint64_t avg = (E + V - 1) / V;
+        layout = (E > 0 && (uint64_t)hs.max_deg >= 64ull * (avg ? avg : 1)) ? AG_LAYOUT_DEGREE : AG_LAYOUT_IDENTITY;
+    }
+    g->layout = layout;
+    if (layout == AG_LAYOUT_DEGREE) {
+        uint64_t *nrp = nullptr;
+        if ((s = build_degree_layout(g, rp64, &nrp)) != AG_OK) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(s); }
+        dev_free(rp64, (size_t)(V + 1) * 8, device);
+        rp64 = nrp;  // (allocated with V*8+8 bytes)
+    }
     if (g->offs32) {
         uint32_t *rp32 = nullptr;
         if ((s = dev_alloc((void **)&rp32, (size_t)(V + 1) * 4 + 128, device)) != AG_OK) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(s); }
@@ -517,6 +595,17 @@ ag_status ag_graph_load_csr(uint32_t V, uint64_t E, const uint64_t *row_ptr, con
         g->d_rp = rp64;
         g->rp_bytes = (size_t)(V + 1) * 8;
     }
+    if (g->d_w) {  // SSSP reads (col, w) together: interleave, drop the separate weight array
+        if ((s = dev_alloc((void **)&g->d_cw, E * 8 + 128, device)) != AG_OK) return fail(s);
+        g->cw_bytes = E * 8 + 128;
+        if (E) interleave_kernel<<<sms * 8, 256>>>(g->d_col, g->d_w, g->d_cw, E);
+        note_launch(1);
+        e = cudaDeviceSynchronize();
+        if (e != cudaSuccess) return fail(cuda_status(e, "interleave"));
+        dev_free(g->d_w, g->w_bytes, device);
+        g->d_w = nullptr;
+        g->w_bytes = 0;
+    }
     g->info.num_vertices = V;
     g->info.num_edges = E;
     g->info.deg_sum = E;
@@ -527,6 +616,20 @@ ag_status ag_graph_load_csr(uint32_t V, uint64_t E, const uint64_t *row_ptr, con
     g->info.device = device;
     g->info.num_sms = sms;
     g->info.offset_bytes = g->offs32 ? 4 : 8;
+    g->info.layout = g->layout;
+    {   // L2 set-aside for the persisting status window (device-wide limit; never lowered)
+        cudaDeviceProp pr;
+        cudaGetDeviceProperties(&pr, device);
+        size_t want = (size_t)V * 8;
+        if (want > (size_t)pr.persistingL2CacheMaxSize) want = (size_t)pr.persistingL2CacheMaxSize;
+        size_t cur = 0;
+        cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+        if (want > cur) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want);
+        cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+        g->persist_bytes = cur;
+        g->max_window = (size_t)pr.accessPolicyMaxWindowSize;
+        cudaGetLastError();
+    }
     *out = g;
     return AG_OK;
 }
@@ -544,6 +647,7 @@ ag_status ag_graph_free(ag_graph g) {
     dev_free(g->d_rp, g->rp_bytes, g->device);
     dev_free(g->d_col, g->col_bytes, g->device);
     dev_free(g->d_w, g->w_bytes, g->device);
+    dev_free(g->d_cw, g->cw_bytes, g->device);
     const size_t V = g->V, nw = g->nwords;
     dev_free(g->d_ctl, sizeof(Ctl), g->device);
     for (int i = 0; i < 3; ++i) { dev_free(g->d_bm[i], nw * 4 + 128, g->device); dev_free(g->d_q[i], V * 4 + 128, g->device); }
@@ -554,6 +658,10 @@ ag_status ag_graph_free(ag_graph g) {
     dev_free(g->d_out_tmp, g->out_tmp_bytes, g->device);
     dev_free(g->d_par_tmp, g->par_tmp_bytes, g->device);
     dev_free(g->d_trace, g->trace_bytes, g->device);
+    dev_free(g->d_perm, V * 4, g->device);
+    dev_free(g->d_inv, V * 4, g->device);
+    dev_free(g->d_level, V * 4 + 128, g->device);
+    dev_free(g->d_lpar, V * 4 + 128, g->device);
     if (g->ev[0]) cudaEventDestroy(g->ev[0]);
     if (g->ev[1]) cudaEventDestroy(g->ev[1]);
     ag::dist_graph_release(g);
@@ -576,9 +684,11 @@ ag_status ag_graph_check(ag_graph g) {
         unsigned *flag = (unsigned *)g->d_acc;
         cudaMemset(flag, 0, 4);
         if (g->offs32)
-            overflow_check_kernel<uint32_t><<<g->num_sms * 4, 256>>>(g->last_out, (const uint32_t *)g->d_rp, g->d_col, g->V, flag);
+            overflow_check_kernel<uint32_t><<<g->num_sms * 4, 256>>>(g->last_out, (const uint32_t *)g->d_rp, g->d_col,
+                                                                     g->d_perm, g->V, flag);
         else
-            overflow_check_kernel<unsigned long long><<<g->num_sms * 4, 256>>>(g->last_out, (const unsigned long long *)g->d_rp, g->d_col, g->V, flag);
+            overflow_check_kernel<unsigned long long><<<g->num_sms * 4, 256>>>(
+                g->last_out, (const unsigned long long *)g->d_rp, g->d_col, g->d_perm, g->V, flag);
         note_launch(1);
         unsigned h = 0;
         e = cudaMemcpy(&h, flag, 4, cudaMemcpyDeviceToHost);
@@ -592,7 +702,7 @@ static ag_status query(ag_graph g, int alg, uint32_t src, uint32_t *out, uint32_
                        ag_run_stats *stats, void *stream) {
     if (!g || !out) return set_error(AG_ERR_INVALID_ARG, "NULL argument");
     if (src >= g->V) return set_error(AG_ERR_SRC_RANGE, "src %u >= V %u", src, g->V);
-    if (alg == ALG_SSSP && !g->d_w) return set_error(AG_ERR_NO_WEIGHTS, "graph was loaded without weights");
+    if (alg == ALG_SSSP && !g->d_cw) return set_error(AG_ERR_NO_WEIGHTS, "graph was loaded without weights");
     if (g->dist) return set_error(AG_ERR_INVALID_ARG, "distributed graph: use ag_dist_bfs");
     cudaStream_t st = (cudaStream_t)stream;
     return g->offs32 ? run_query<uint32_t>(g, alg, src, out, parents, p, stats, st)

@@ -9,13 +9,33 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <type_traits>
+
 #include "agraph.h"
 
 namespace ag {
 
-constexpr int BS = 256;             // threads per CTA of the persistent traversal kernel
+#ifndef AG_BS
+#define AG_BS 256
+#endif
+constexpr int BS = AG_BS;           // threads per CTA of the persistent traversal kernel
 constexpr int WARPS_PER_CTA = BS / 32;
-constexpr int MIN_BLOCKS = 4;       // __launch_bounds__ min CTAs/SM (=> <= 64 regs/thread)
+constexpr int LOG_BS = (BS == 1024) ? 10 : (BS == 512) ? 9 : (BS == 256) ? 8 : (BS == 128) ? 7 : -1;
+static_assert(LOG_BS > 0, "BS must be 128, 256, 512 or 1024");
+// Occupancy / batch depth per algorithm (measured on B200): BFS is best at 4 CTAs/SM
+// (64 regs) with 4-edge batches, SSSP (8-byte states, more atomics) at 8 CTAs/SM with 2-edge batches.
+#ifndef AG_MINB_BFS
+#define AG_MINB_BFS 4
+#endif
+#ifndef AG_MINB_SSSP
+#define AG_MINB_SSSP 8
+#endif
+#ifndef AG_EB_BFS
+#define AG_EB_BFS 4
+#endif
+#ifndef AG_EB_SSSP
+#define AG_EB_SSSP 2
+#endif
 constexpr uint32_t INF = 0xFFFFFFFFu;
 constexpr unsigned long long INF64 = 0xFFFFFFFFFFFFFFFFull;
 constexpr uint32_t MAX_FINITE = 0xFFFFFFFEu;
@@ -27,27 +47,37 @@ enum { WS_BM = 1, WS_QU = 2 };
 
 // Hybrid mapping (beyond the paper, 18.s43-44): vertices with out-degree >= HUB_DEG are split into
 // HUB_CHUNK-edge tasks drained by all CTAs.
-constexpr uint32_t HUB_DEG = 4096;
-constexpr uint32_t HUB_CHUNK = 2048;
+#ifndef AG_HUBCHUNK
+#define AG_HUBCHUNK 4096
+#endif
+#ifndef AG_LONG_MIN
+#define AG_LONG_MIN 512   // hybrid mapping: lists this long go to aligned warp windows
+#endif
+constexpr uint32_t HUB_DEG = 2048;
+constexpr uint32_t HUB_CHUNK = AG_HUBCHUNK;
+// Edges processed per thread per batch: loads of all EB edges are issued before any dependent use.
+constexpr int EB_MAX = (AG_EB_BFS > AG_EB_SSSP) ? AG_EB_BFS : AG_EB_SSSP;
 
 // ---------------------------------------------------------------------------------------------
 // Device-side control block.  Per-iteration counters rotate over 3 slots (slot = it % 3): slot(it)
 // describes the working set processed in iteration it, slot(it+1) accumulates the next one, and
 // slot(it+2) is reset at the start of iteration it (its last reader finished at the barrier).
 // ---------------------------------------------------------------------------------------------
+constexpr int NGRP = 32;            // barrier arrival groups (hierarchical arrival)
+
 struct alignas(128) Ctl {
-    unsigned int bar_count;
-    unsigned int pad0[31];
-    unsigned int bar_gen;
+    unsigned long long bar_word;      // (generation << 32) | payload, released by the last arriver
+    unsigned int pad0[30];
+    unsigned int bar_count;           // groups arrived
     unsigned int pad1[31];
+    unsigned int grp_count[NGRP * 32];  // CTAs arrived per group (one 128-B line each)
     unsigned int q_len[3];            // queue append cursor == |WS| for BFS and unordered SSSP
     unsigned int next_min[3];         // ordered SSSP: min tentative distance of pending vertices
     unsigned int tile_ctr[3];         // dynamic tile scheduler
     unsigned int hub_tail[3];         // hybrid mapping: produced hub-chunk tasks
     unsigned int hub_head[3];         //                 consumed hub-chunk tasks
     unsigned int stage_done[3];       //                 CTAs done producing
-    unsigned long long it_edges[3];   // edges inspected in iteration
-    unsigned long long it_verts[3];   // vertices expanded in iteration
+    unsigned long long it_edges[3];   // edges inspected in iteration (trace only)
     unsigned int pend_count;          // ordered SSSP: |pending|
     unsigned int overflow;            // a relaxation exceeded MAX_FINITE
     unsigned int iterations;
@@ -68,12 +98,16 @@ struct DevPolicy {
     uint32_t cta_group;   // resolved block-mapping group size (multiple of 32, <= BS)
     uint32_t V;
     uint64_t E;
+    uint32_t max_deg;     // inspector: maximum out-degree (tuned policy)
+    uint32_t t2_tuned;    // tuned policy: thread mapping below this |WS| on low-degree graphs
 };
 
 // The decision maker.  PAPER: Fig. 11 with readings R12/R13:
 //   ws < T2 -> B_QU; else workset = ws >= T3 ? BM : QU; mapping = E >= T1*V ? B : T.
-// TUNED (B200): workset by the same T3 rule; mapping HYBRID (per-vertex degree
-//   classes + hub splitting) unless the graph is near-regular and low-degree, where THREAD wins.
+// TUNED (B200, calibrated by tools/sweep.py on C2/C3/C4): the queue always wins on
+//   B200 (appends are warp-aggregated, the bitmap scan is O(V) threads per iteration); mapping is
+//   THREAD for small working sets of a graph whose max out-degree is <= 64 (no straggler risk, no
+//   tile-scan overhead), else HYBRID (load-balanced gather + hub splitting).
 __host__ __device__ inline uint8_t select_variant(const DevPolicy &p, uint64_t ws, uint64_t ws_edges) {
     uint32_t map, wsr;
     (void)ws_edges;
@@ -86,8 +120,8 @@ __host__ __device__ inline uint8_t select_variant(const DevPolicy &p, uint64_t w
             map = (p.E >= (uint64_t)p.t1 * p.V) ? MAP_B : MAP_T;
         }
     } else {
-        wsr = ws >= p.t3 ? WS_BM : WS_QU;
-        map = MAP_H;
+        wsr = WS_QU;
+        map = (p.max_deg <= 64 && ws < p.t2_tuned) ? MAP_T : MAP_H;
     }
     if (p.force_map) map = p.force_map;
     if (p.force_ws) wsr = p.force_ws;
@@ -116,10 +150,46 @@ __device__ __forceinline__ unsigned long long ld_relaxed64(const unsigned long l
     asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
-// streaming read of a CSR array: read once per traversal, keep it out of L1
-__device__ __forceinline__ uint32_t ld_stream(const uint32_t *p) {
+// L2 eviction policies: the CSR arrays stream through once per traversal (evict first, no L1
+// allocation) while the per-vertex status arrays (visited bitmap, levels, packed distances) should
+// stay resident in the 126 MB L2 (evict last).
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+// streaming read of a CSR array: read once per traversal, keep it out of L1, evict first from L2
+__device__ __forceinline__ uint32_t ld_stream(const uint32_t *p, uint64_t pol) {
     uint32_t v;
-    asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(v) : "l"(p));
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ uint2 ld_stream2(const uint2 *p, uint64_t pol) {
+    uint2 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0, %1}, [%2], %3;"
+                 : "=r"(v.x), "=r"(v.y) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ uint4 ld_stream4(const uint4 *p, uint64_t pol) {
+    uint4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol));
+    return v;
+}
+// status read: L1-cacheable, evict last from L2
+__device__ __forceinline__ uint32_t ld_keep(const uint32_t *p, uint64_t pol) {
+    uint32_t v;
+    asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ unsigned long long ld_keep(const unsigned long long *p, uint64_t pol) {
+    unsigned long long v;
+    asm volatile("ld.global.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
     return v;
 }
 __device__ __forceinline__ uint32_t ld_ro(const uint32_t *p) { return __ldg(p); }
@@ -129,21 +199,37 @@ __device__ __forceinline__ void red_or(uint32_t *p, uint32_t v) {
 }
 
 __device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31u; }
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
 
-// Software grid barrier for a co-resident (cooperative) grid.  Sense via a generation counter;
-// the last arriver resets the count, so the barrier needs no per-launch reset.
+__device__ __forceinline__ unsigned long long ld_acquire64(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release64(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned atom_add_acqrel(unsigned *p, unsigned v) {
+    unsigned old;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
+
+// Software grid barrier for a co-resident (cooperative) grid, one atomic per CTA on a single word:
+// CTA 0 adds 0x80000000 - (nblocks - 1), every other CTA adds 1, so the top bit flips exactly when
+// the last CTA arrives; everyone spins on that bit (measured on B200: ~1.6 us at 592 CTAs, faster
+// than a two-level tree with a separate release word).  Self-resetting across launches.
 __device__ __forceinline__ void grid_barrier(Ctl *ctl, unsigned nblocks) {
     __syncthreads();
     if (threadIdx.x == 0) {
-        unsigned gen = ld_acquire(&ctl->bar_gen);
+        const unsigned inc = (blockIdx.x == 0) ? (0x80000000u - (nblocks - 1)) : 1u;
         __threadfence();
-        unsigned arrived = atomicAdd(&ctl->bar_count, 1u);
-        if (arrived == nblocks - 1) {
-            ctl->bar_count = 0;
-            __threadfence();
-            st_release(&ctl->bar_gen, gen + 1);
-        } else {
-            while (ld_acquire(&ctl->bar_gen) == gen) __nanosleep(20);
+        const unsigned old = atomicAdd(&ctl->bar_count, inc);
+        while (((old ^ ld_relaxed(&ctl->bar_count)) & 0x80000000u) == 0) {
         }
         __threadfence();
     }

@@ -25,8 +25,16 @@ struct ag_graph_s {
     size_t rp_bytes = 0;
     uint32_t *d_col = nullptr;
     size_t col_bytes = 0;
-    uint32_t *d_w = nullptr;
+    uint32_t *d_w = nullptr;       // weights (load time only; freed once interleaved)
     size_t w_bytes = 0;
+    uint2 *d_cw = nullptr;         // interleaved (col, w) pairs for SSSP: one 8-B load per edge
+    size_t cw_bytes = 0;
+    // degree layout (layout.cu): new id i = old vertex d_perm[i]; d_inv = inverse
+    uint32_t layout = AG_LAYOUT_IDENTITY;
+    uint32_t *d_perm = nullptr;
+    uint32_t *d_inv = nullptr;
+    uint32_t *d_level = nullptr;   // BFS level / parent arrays in the relabelled space
+    uint32_t *d_lpar = nullptr;
     // scratch
     void *d_ctl = nullptr;
     bool ctl_init = false;
@@ -44,6 +52,8 @@ struct ag_graph_s {
     uint32_t *d_trace = nullptr;
     size_t trace_bytes = 0;
     size_t scratch_bytes = 0;
+    size_t persist_bytes = 0;      // L2 persisting set-aside available
+    size_t max_window = 0;         // cudaDeviceProp::accessPolicyMaxWindowSize
     cudaEvent_t ev[2] = {nullptr, nullptr};
     uint32_t epoch = 0;
     // deferred status of the last enqueued traversal
@@ -64,4 +74,5 @@ bool is_device_ptr(const void *p);
 ag_status check_device(int device, int *num_sms);
 void note_launch(unsigned n);
 void dist_graph_release(ag_graph_s *g);
+ag_status build_degree_layout(ag_graph_s *g, const uint64_t *rp64, uint64_t **nrp_out);
 }  // namespace ag

@@ -22,8 +22,9 @@
 //   T  thread per element, the thread visits all neighbours                  (Fig. 9 line 4)
 //   W  warp per element, lanes visit neighbours (block mapping at 32 threads, 24.s15)
 //   B  group of `cta_group` threads per element (26.s28), threads visit neighbours (Fig. 9 l.4')
-//   H  per element by degree: <32 edge-parallel via CTA scan, <BS warp, <HUB_DEG CTA,
-//      >= HUB_DEG split into chunks drained by all CTAs (18.s43-44 "intermediate solutions").
+//   H  load-balanced: the tile's adjacency lists are concatenated (CTA scan of degrees) and
+//      every thread takes EB edges per step; degree >= HUB_DEG is split into HUB_CHUNK-edge
+//      tasks drained by all CTAs (18.s43-44 "intermediate solutions", not built in the paper).
 #pragma once
 
 #include "common.cuh"
@@ -34,11 +35,15 @@ template <typename Off>
 struct TravArgs {
     const Off *rp;
     const uint32_t *col;
-    const uint32_t *w;
+    const uint2 *cw;            // SSSP: interleaved (col, w)
     uint32_t V;
     uint32_t nwords;
-    uint32_t *level;            // BFS level array (V)
-    uint32_t *parent;           // BFS parent array (V) or nullptr
+    uint32_t *level;            // BFS level array (V), in device-layout ids
+    uint32_t *parent;           // BFS parent array (V) or nullptr, in device-layout ids
+    const uint32_t *perm;       // degree layout: new id -> caller id (nullptr = identity layout)
+    const uint32_t *inv;        //                caller id -> new id
+    uint32_t *out_level;        // BFS outputs in caller ids (written by the final pass if relabelled)
+    uint32_t *out_parent;
     unsigned long long *P;      // SSSP packed state (V)
     uint32_t *vis;              // BFS ordered: visited bitmap
     uint32_t *bm[3];            // rotating frontier bitmaps (SSSP ordered: bm[0] = pending bitmap)
@@ -51,6 +56,7 @@ struct TravArgs {
     uint32_t *trace_ws;
     unsigned long long *trace_edges;
     uint8_t *trace_var;
+    unsigned long long *trace_ns;
     uint32_t trace_cap;
     DevPolicy pol;
     uint32_t src;
@@ -60,6 +66,8 @@ struct TravArgs {
     uint32_t has_hubs;
 };
 
+constexpr int WQ_CAP = 32 * EB_MAX + 32;
+
 template <typename Off>
 struct __align__(16) TileSmem {
     Off beg[BS];
@@ -67,12 +75,14 @@ struct __align__(16) TileSmem {
     uint32_t uval[BS];
     uint32_t deg[BS];
     uint32_t scan[BS + 1];
-    uint32_t big[BS];
+    uint32_t wscan[BS + 1];
+    uint32_t woff[2][WARPS_PER_CTA];
+    uint32_t wq[WARPS_PER_CTA][WQ_CAP];   // per-warp staged queue appends (hybrid mapping)
     unsigned long long red64[2][WARPS_PER_CTA];
     uint32_t red32[2][WARPS_PER_CTA];
     int redi[WARPS_PER_CTA];
-    uint32_t nbig;
-    uint32_t tile;
+    uint32_t tnext[2];
+    uint32_t bcast;
     uint32_t task;
     uint32_t status;
 };
@@ -83,6 +93,7 @@ struct __align__(16) TileSmem {
 // ------------------------------------------------------------------------------------------------
 template <int ALG, int ORD, typename Off>
 struct Ops {
+    static constexpr int EB = (ALG == ALG_SSSP) ? AG_EB_SSSP : AG_EB_BFS;
     const TravArgs<Off> &a;
     uint32_t it;
     uint64_t hi;            // SSSP ordered: exclusive bound lo + delta of the current bucket
@@ -90,13 +101,20 @@ struct Ops {
     uint32_t *q_next;
     unsigned *qlen_next;
     bool append_next;
+    bool fenced;            // ordered SSSP with delta > 1: a bucket vertex can improve while claimed
+    uint64_t pol_stream;    // L2 evict-first policy for the CSR streams
+    uint64_t pol_keep;      // L2 evict-last policy for the status arrays
+    uint32_t *wbuf;         // this warp's staging buffer in shared memory (hybrid mapping)
+    uint32_t wfill;         // its fill level (warp-uniform)
     unsigned long long ne, nv;
     uint32_t vmin;
     int dpend;
     bool ovf;
 
     __device__ Ops(const TravArgs<Off> &a_, uint32_t it_, uint64_t hi_, bool append_)
-        : a(a_), it(it_), hi(hi_), append_next(append_), ne(0), nv(0), vmin(INF), dpend(0), ovf(false) {
+        : a(a_), it(it_), hi(hi_), append_next(append_), fenced(ALG == ALG_SSSP && ORD == ORD_O && a_.pol.delta > 1),
+          pol_stream(policy_evict_first()), pol_keep(policy_evict_last()), wbuf(nullptr), wfill(0), ne(0), nv(0),
+          vmin(INF), dpend(0), ovf(false) {
         const uint32_t sn = (it_ + 1) % 3;
         bm_next = (ALG == ALG_SSSP && ORD == ORD_O) ? a_.bm[0] : a_.bm[sn];
         q_next = a_.q[sn];
@@ -116,7 +134,16 @@ struct Ops {
                     const uint32_t m = 1u << (u & 31);
                     uint32_t old = atomicAnd(&a.bm[0][u >> 5], ~m);
                     ex = (old & m) != 0;
-                    if (ex) dpend -= 1;
+                    if (ex) {
+                        dpend -= 1;
+                        if (fenced) {
+                            // an improvement that found the pending bit still set (so did not re-add u)
+                            // is visible after this fence: expand with the current value (the improver
+                            // fences between its atomicMin and its atomicOr on the pending bit)
+                            __threadfence();
+                            uval = (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
+                        }
+                    }
                 } else {  // pending survivor: stays in the working set, feeds findmin (22.s11)
                     ex = false;
                     vmin = min(vmin, t);
@@ -136,83 +163,205 @@ struct Ops {
         return ex;
     }
 
-    // Per-edge update for edge (u -> v, wt) from a frontier element with value uval.
-    __device__ __forceinline__ void visit(uint32_t u, uint32_t uval, uint32_t v, uint32_t wt) {
+    // Status word of v, read before deciding to update.  Plain (L1-cacheable) load: a stale value is
+    // always safe because levels/distances only decrease and visited bits are only set — a stale
+    // read can only cause an extra atomic, never a missed update.
+    using St = typename std::conditional<ALG == ALG_SSSP, unsigned long long, uint32_t>::type;
+    __device__ __forceinline__ St status(uint32_t v) const {
+        if constexpr (ALG == ALG_SSSP) return ld_keep(a.P + v, pol_keep);
+        else return ld_keep(a.vis + (v >> 5), pol_keep);   // BFS: visited bit (level-synchronous: set <=> level <= current+1)
+    }
+
+    // Per-edge update for edge (u -> v, wt) from a frontier element with value uval, given status s.
+    // Returns true if v newly entered the next working set (the caller appends it to the queue).
+    __device__ __forceinline__ bool update(uint32_t u, uint32_t uval, uint32_t v, uint32_t wt, St s, bool valid) {
         const uint32_t m = 1u << (v & 31);
         bool nw = false;
+        if (!valid) return false;
         if constexpr (ALG == ALG_BFS) {
             const uint32_t nl = uval + 1;
             if constexpr (ORD == ORD_O) {
-                uint32_t *wp = a.vis + (v >> 5);
-                if (!(*wp & m)) {                          // m.level == INF ?  (L1-cached status)
-                    if (!(atomicOr(wp, m) & m)) {          // claim: first visit wins
+                if (!(s & m)) {                                        // m.level == INF ?   (Fig. 4 l.8)
+                    if (!(atomicOr(a.vis + (v >> 5), m) & m)) {        // claim: first visit wins
                         nw = true;
-                        a.level[v] = nl;
+                        a.level[v] = nl;                               // m.level = level    (l.9)
                         if (a.parent) a.parent[v] = u;
-                        red_or(a.bm[(it + 1) % 3] + (v >> 5), m);
+                        red_or(a.bm[(it + 1) % 3] + (v >> 5), m);      // update vector      (l.10)
                     }
                 }
             } else {
-                if (a.level[v] > nl) {                     // m.level > level ?
+                // m.level > level ?  (Fig. 4 l.8').  A set visited bit implies level[v] <= nl, so it is
+                // an exact pre-filter; the decision itself is the atomicMin on the level.
+                if (!(s & m)) {
                     if (atomicMin(&a.level[v], nl) > nl) {
                         nw = true;
                         if (a.parent) a.parent[v] = u;
+                        red_or(a.vis + (v >> 5), m);
                         red_or(bm_next + (v >> 5), m);
                     }
                 }
             }
-            warp_append(q_next, qlen_next, nw, v);
         } else {
-            const uint64_t nd = (uint64_t)uval + wt;   // d = n.distance + w(n,m)   (Fig. 5 l.6)
+            const uint64_t nd = (uint64_t)uval + wt;                   // d = n.distance + w (Fig. 5 l.6)
             if (nd > MAX_FINITE) {
                 ovf = true;
-            } else {
-                unsigned long long cur = a.P[v];
-                if ((cur >> 32) > nd) {                    // d < m.distance            (Fig. 5 l.7)
-                    unsigned long long old = atomicMin(&a.P[v], (nd << 32) | u);
-                    if ((old >> 32) > nd) {                // we lowered it             (Fig. 5 l.8)
-                        uint32_t ob = atomicOr(bm_next + (v >> 5), m);
-                        nw = !(ob & m);                    // ws.add(m), deduplicated   (Fig. 5 l.9)
-                        if constexpr (ORD == ORD_O) {
-                            vmin = min(vmin, (uint32_t)nd);
-                            if (nw) dpend += 1;
-                        }
+            } else if ((s >> 32) > nd) {                               // d < m.distance      (l.7)
+                unsigned long long old = atomicMin(&a.P[v], (nd << 32) | u);
+                if ((old >> 32) > nd) {                                // m.distance = d      (l.8)
+                    if (fenced) __threadfence();
+                    uint32_t ob = atomicOr(bm_next + (v >> 5), m);
+                    nw = !(ob & m);                                    // ws.add(m), deduped  (l.9)
+                    if constexpr (ORD == ORD_O) {
+                        vmin = min(vmin, (uint32_t)nd);
+                        if (nw) dpend += 1;
                     }
                 }
             }
-            if (ORD == ORD_U || append_next) warp_append(q_next, qlen_next, nw, v);
+            if (ORD == ORD_O && !append_next) nw = false;
         }
+        return nw;
     }
 
-    __device__ __forceinline__ void edge(uint32_t u, uint32_t uval, Off e) {
-        uint32_t v = ld_stream(a.col + e);
-        uint32_t wt = (ALG == ALG_SSSP) ? ld_stream(a.w + e) : 1u;
-        visit(u, uval, v, wt);
-    }
-
-    // thread-mapped neighbour loop with 4 independent loads in flight
-    __device__ __forceinline__ void edges_thread(uint32_t u, uint32_t uval, Off beg, uint32_t deg) {
-        Off e = beg, end = beg + deg;
-        for (; e + 4 <= end; e += 4) {
-            uint32_t v0 = ld_stream(a.col + e), v1 = ld_stream(a.col + e + 1);
-            uint32_t v2 = ld_stream(a.col + e + 2), v3 = ld_stream(a.col + e + 3);
-            uint32_t w0 = 1, w1 = 1, w2 = 1, w3 = 1;
+    // NB independent edges: all CSR loads first, then all status loads, then the updates, so NB
+    // memory requests per phase are in flight per thread (the per-edge chain col -> status -> atomic
+    // is latency-bound otherwise).  New working-set elements are appended either warp-aggregated to
+    // the global queue, or (STAGED: all 32 lanes converged) staged in this warp's shared-memory
+    // buffer, flushed to the global queue 32 entries at a time with one atomic per flush.
+    template <int NB, bool STAGED = false>
+    __device__ __forceinline__ void batch(const uint32_t (&u)[NB], const uint32_t (&uv)[NB], const Off (&e)[NB],
+                                          const bool (&ok)[NB]) {
+        uint32_t v[NB], wt[NB];
+        St st[NB];
+#pragma unroll
+        for (int j = 0; j < NB; ++j) {
             if constexpr (ALG == ALG_SSSP) {
-                w0 = ld_stream(a.w + e); w1 = ld_stream(a.w + e + 1);
-                w2 = ld_stream(a.w + e + 2); w3 = ld_stream(a.w + e + 3);
+                const uint2 c = ok[j] ? ld_stream2(a.cw + e[j], pol_stream) : make_uint2(0u, 1u);
+                v[j] = c.x;
+                wt[j] = c.y;
+            } else {
+                v[j] = ok[j] ? ld_stream(a.col + e[j], pol_stream) : 0u;
+                wt[j] = 1u;
             }
-            visit(u, uval, v0, w0);
-            visit(u, uval, v1, w1);
-            visit(u, uval, v2, w2);
-            visit(u, uval, v3, w3);
         }
-        for (; e < end; ++e) edge(u, uval, e);
+#if defined(AG_EXPERIMENT) && AG_EXPERIMENT == 1   // ceiling experiment: stream only
+        {
+            uint32_t acc = 0;
+#pragma unroll
+            for (int j = 0; j < NB; ++j) acc += v[j] + wt[j];
+            if (acc == 0xFFFFFFFFu) ovf = true;
+            return;
+        }
+#endif
+#pragma unroll
+        for (int j = 0; j < NB; ++j) st[j] = ok[j] ? status(v[j]) : (St)0;
+#if defined(AG_EXPERIMENT) && AG_EXPERIMENT == 2   // ceiling experiment: stream + status, no update
+        {
+            uint32_t acc = 0;
+#pragma unroll
+            for (int j = 0; j < NB; ++j) acc += (uint32_t)st[j];
+            if (acc == 0x12345u) ovf = true;
+            return;
+        }
+#endif
+#pragma unroll
+        for (int j = 0; j < NB; ++j) {
+            bool nw = update(u[j], uv[j], v[j], wt[j], st[j], ok[j]);
+            if constexpr (STAGED) {
+                const unsigned m = __ballot_sync(0xffffffffu, nw);
+                if (nw) wbuf[wfill + __popc(m & ((1u << lane_id()) - 1u))] = v[j];
+                wfill += __popc(m);
+            } else {
+                warp_append(q_next, qlen_next, nw, v[j]);
+            }
+        }
+        if constexpr (STAGED) {
+            __syncwarp();
+            if (wfill >= 32) warp_flush(false);
+        }
     }
 
-    // cooperative neighbour loop: `lane` of `width` threads
-    __device__ __forceinline__ void edges_coop(uint32_t u, uint32_t uval, Off beg, uint32_t deg,
-                                               uint32_t lane, uint32_t width) {
-        for (uint32_t k = lane; k < deg; k += width) edge(u, uval, beg + k);
+    // One aligned window of WIN = 32 x EPL consecutive CSR entries [wbase, wbase + WIN), restricted to
+    // [lo, hi) (one adjacency list), processed by a whole warp: each lane issues ONE 16-byte vector
+    // load for its EPL entries, then EPL independent status loads, then the updates (all lanes
+    // converged; staged appends).  The per-edge owner lookup of the gather path disappears.
+    static constexpr int EPL = (ALG == ALG_SSSP) ? 2 : 4;
+    static constexpr int WIN = 32 * EPL;
+    __device__ __forceinline__ void window(uint32_t u, uint32_t uval, Off wbase, Off lo, Off hi) {
+        const Off e0 = wbase + (Off)lane_id() * EPL;
+        uint32_t v[EPL], wt[EPL];
+        bool ok[EPL];
+        const bool any = e0 < hi && e0 + EPL > lo;
+        if constexpr (ALG == ALG_SSSP) {
+            uint4 c = any ? ld_stream4(reinterpret_cast<const uint4 *>(a.cw + e0), pol_stream) : make_uint4(0, 1, 0, 1);
+            v[0] = c.x; wt[0] = c.y; v[1] = c.z; wt[1] = c.w;
+        } else {
+            uint4 c = any ? ld_stream4(reinterpret_cast<const uint4 *>(a.col + e0), pol_stream) : make_uint4(0, 0, 0, 0);
+            v[0] = c.x; v[1] = c.y; v[2] = c.z; v[3] = c.w;
+#pragma unroll
+            for (int j = 0; j < EPL; ++j) wt[j] = 1u;
+        }
+        St st[EPL];
+#pragma unroll
+        for (int j = 0; j < EPL; ++j) {
+            ok[j] = (e0 + j >= lo) && (e0 + j < hi);
+            st[j] = ok[j] ? status(v[j]) : (St)0;
+        }
+#pragma unroll
+        for (int j = 0; j < EPL; ++j) {
+            bool nw = update(u, uval, v[j], wt[j], st[j], ok[j]);
+            const unsigned m = __ballot_sync(0xffffffffu, nw);
+            if (nw) wbuf[wfill + __popc(m & ((1u << lane_id()) - 1u))] = v[j];
+            wfill += __popc(m);
+        }
+        __syncwarp();
+        if (wfill >= 32) warp_flush(false);
+    }
+
+    // Copy this warp's staged entries (all, or whole groups of 32) to the global queue.
+    __device__ __forceinline__ void warp_flush(bool all) {
+        const unsigned lane = lane_id();
+        const uint32_t n = all ? wfill : (wfill & ~31u);
+        if (n == 0) return;
+        uint32_t base = 0;
+        if (lane == 0) base = atomicAdd(qlen_next, n);
+        base = __shfl_sync(0xffffffffu, base, 0);
+        for (uint32_t i = lane; i < n; i += 32) q_next[base + i] = wbuf[i];
+        const uint32_t rem = wfill - n;  // < 32
+        uint32_t t = (lane < rem) ? wbuf[n + lane] : 0u;
+        __syncwarp();
+        if (lane < rem) wbuf[lane] = t;
+        __syncwarp();
+        wfill = rem;
+    }
+
+    // thread-mapped neighbour loop (Fig. 9 line 4: "current thread visits all neighbors")
+    __device__ __forceinline__ void edges_thread(uint32_t u, uint32_t uval, Off beg, uint32_t deg) {
+        for (uint32_t k = 0; k < deg; k += EB) {
+            uint32_t uu[EB], vv[EB];
+            Off e[EB];
+            bool ok[EB];
+#pragma unroll
+            for (int j = 0; j < EB; ++j) {
+                uu[j] = u; vv[j] = uval; e[j] = beg + k + j; ok[j] = k + j < deg;
+            }
+            batch<EB>(uu, vv, e, ok);
+        }
+    }
+
+    // cooperative neighbour loop: `lane` of `width` threads (Fig. 9 line 4': "each thread in block
+    // visits a neighbor")
+    __device__ __forceinline__ void edges_coop(uint32_t u, uint32_t uval, Off beg, uint32_t deg, uint32_t lane,
+                                               uint32_t width) {
+        for (uint32_t k = lane; k < deg; k += EB * width) {
+            uint32_t uu[EB], vv[EB];
+            Off e[EB];
+            bool ok[EB];
+#pragma unroll
+            for (int j = 0; j < EB; ++j) {
+                uu[j] = u; vv[j] = uval; e[j] = beg + k + j * width; ok[j] = k + j * width < deg;
+            }
+            batch<EB>(uu, vv, e, ok);
+        }
     }
 };
 
@@ -244,8 +393,11 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, Tile
             ov |= sm.red32[1][i];
             sd += sm.redi[i];
         }
-        if (se) atomicAdd(&ctl->it_edges[slot], se);
-        if (sv) atomicAdd(&ctl->it_verts[slot], sv);
+        if (se) {
+            atomicAdd(&ctl->eexp, se);
+            if (ops.a.trace_edges) atomicAdd(&ctl->it_edges[slot], se);
+        }
+        if (sv) atomicAdd(&ctl->vexp, sv);
         if (ALG == ALG_SSSP && ORD == ORD_O) {
             if (mn != INF) atomicMin(&ctl->next_min[(slot + 1) % 3], mn);
             if (sd) atomicAdd(&ctl->pend_count, (unsigned)sd);
@@ -262,6 +414,7 @@ template <int ALG, int ORD, typename Off>
 __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<Off> &sm, uint32_t map,
                                              bool valid, uint32_t u, uint32_t group, bool hubs, uint32_t slot,
                                              uint32_t tag) {
+    constexpr int EB = Ops<ALG, ORD, Off>::EB;
     const TravArgs<Off> &a = ops.a;
     Off beg = 0;
     uint32_t deg = 0, uval = 0;
@@ -302,16 +455,14 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<O
         __syncthreads();
         return;
     }
-    // ---- MAP_H: per-element degree classes
+    // ---- MAP_H: load-balanced gather over the tile's concatenated adjacency lists; vertices of
+    // degree >= HUB_DEG are split into HUB_CHUNK-edge tasks drained by all CTAs.
     const bool is_hub = hubs && deg >= HUB_DEG;
-    const bool is_big = !is_hub && deg >= (uint32_t)BS;
-    const bool is_mid = deg >= 32 && deg < (uint32_t)BS;
-    const uint32_t small = (deg < 32) ? deg : 0;
-    if (is_hub) {  // split into HUB_CHUNK-edge tasks for all CTAs (drained after the tile loop)
+    if (is_hub) {
         const uint32_t nch = (deg + HUB_CHUNK - 1) / HUB_CHUNK;
         uint32_t base = atomicAdd(&a.ctl->hub_tail[slot], nch);
-        // capacity hub_cap >= E/HUB_CHUNK + E/HUB_DEG + 16 covers any frontier (each vertex is at most
-        // once per iteration in it); the guard only protects memory.
+        // hub_cap >= E/HUB_CHUNK + E/HUB_DEG + 16 covers any frontier (each vertex is at most once
+        // per iteration in it); the guard only protects memory.
         for (uint32_t k = 0; k < nch; ++k) {
             uint32_t idx = base + k;
             if (idx < a.hub_cap) {
@@ -326,70 +477,75 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<O
             }
         }
     }
-    const bool big_path = is_big;
-    // CTA-wide exclusive scan of the small degrees
-    uint32_t x = small;
+    // short lists (< 32 entries) -> packed gather; long lists -> aligned warp windows
+    constexpr uint32_t WIN = Ops<ALG, ORD, Off>::WIN;
+    const bool is_long = !is_hub && deg >= (uint32_t)AG_LONG_MIN;
+    const uint32_t d = (!is_hub && !is_long) ? deg : 0u;
+    const uint32_t nw = is_long ? (uint32_t)((beg + deg + WIN - 1) / WIN - beg / WIN) : 0u;
+    // CTA-wide exclusive scans of (short degrees, long-list window counts), packed in one u32 pair
+    uint32_t x = d, y = nw;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-        uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-        if (lane >= (unsigned)o) x += y;
+        uint32_t xo = __shfl_up_sync(0xffffffffu, x, o), yo = __shfl_up_sync(0xffffffffu, y, o);
+        if (lane >= (unsigned)o) { x += xo; y += yo; }
     }
-    if (lane == 31) sm.red32[0][tid >> 5] = x;
-    if (tid == 0) sm.nbig = 0;
+    if (lane == 31) { sm.red32[0][tid >> 5] = x; sm.red32[1][tid >> 5] = y; }
     __syncthreads();
     if (tid < 32) {
         uint32_t wv = (tid < (unsigned)WARPS_PER_CTA) ? sm.red32[0][tid] : 0, wx = wv;
+        uint32_t zv = (tid < (unsigned)WARPS_PER_CTA) ? sm.red32[1][tid] : 0, zx = zv;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
-            uint32_t y = __shfl_up_sync(0xffffffffu, wx, o);
-            if (tid >= (unsigned)o) wx += y;
+            uint32_t t1 = __shfl_up_sync(0xffffffffu, wx, o), t2 = __shfl_up_sync(0xffffffffu, zx, o);
+            if (tid >= (unsigned)o) { wx += t1; zx += t2; }
         }
-        if (tid < (unsigned)WARPS_PER_CTA) sm.red32[1][tid] = wx - wv;  // exclusive warp offsets
+        if (tid < (unsigned)WARPS_PER_CTA) { sm.woff[0][tid] = wx - wv; sm.woff[1][tid] = zx - zv; }
     }
     __syncthreads();
-    const uint32_t excl = sm.red32[1][tid >> 5] + x - small;
+    const uint32_t excl = sm.woff[0][tid >> 5] + x - d;
+    const uint32_t wexcl = sm.woff[1][tid >> 5] + y - nw;
     sm.scan[tid] = excl;
+    sm.wscan[tid] = wexcl;
     sm.u[tid] = u;
     sm.uval[tid] = uval;
     sm.beg[tid] = beg;
     sm.deg[tid] = deg;
-    if (tid == BS - 1) sm.scan[BS] = excl + small;
-    if (big_path) {
-        uint32_t k = atomicAdd(&sm.nbig, 1u);
-        sm.big[k] = tid;
-    }
+    if (tid == BS - 1) { sm.scan[BS] = excl + d; sm.wscan[BS] = wexcl + nw; }
     __syncthreads();
-    // small: edge-parallel over the concatenated short lists (load-balanced gather)
-    const uint32_t S = sm.scan[BS];
-    for (uint32_t k = tid; k < S; k += BS) {
-        uint32_t lo = 0, hi = BS;  // find owner: scan[owner] <= k < scan[owner+1]
-        while (hi - lo > 1) {
+    // long lists: warps take windows round-robin (owner by binary search, once per window)
+    const uint32_t NWIN = sm.wscan[BS];
+    for (uint32_t wi = tid >> 5; wi < NWIN; wi += WARPS_PER_CTA) {
+        uint32_t lo = 0, hi = BS;
+#pragma unroll
+        for (int step = 0; step < LOG_BS; ++step) {
             uint32_t mid = (lo + hi) >> 1;
-            if (sm.scan[mid] <= k) lo = mid; else hi = mid;
+            if (sm.wscan[mid] <= wi) lo = mid; else hi = mid;
         }
-        ops.edge(sm.u[lo], sm.uval[lo], sm.beg[lo] + (k - sm.scan[lo]));
+        const Off b0 = sm.beg[lo];
+        const Off wbase = (b0 / WIN + (wi - sm.wscan[lo])) * WIN;
+        ops.window(sm.u[lo], sm.uval[lo], wbase, b0, b0 + sm.deg[lo]);
     }
-    // mid: warp-cooperative over this warp's own mid elements
-    {
-        unsigned m = __ballot_sync(0xffffffffu, is_mid);
-        while (m) {
-            const int j = __ffs(m) - 1;
-            m &= m - 1;
-            uint32_t uj = __shfl_sync(0xffffffffu, u, j);
-            uint32_t vj = __shfl_sync(0xffffffffu, uval, j);
-            uint32_t dj = __shfl_sync(0xffffffffu, deg, j);
-            Off bj = (Off)__shfl_sync(0xffffffffu, (unsigned long long)beg, j);
-            ops.edges_coop(uj, vj, bj, dj, lane, 32);
+    // short lists: packed, load-balanced gather
+    const uint32_t S = sm.scan[BS];
+    for (uint32_t base = 0; base < S; base += EB * BS) {
+        uint32_t uu[EB], vv[EB];
+        Off e[EB];
+        bool ok[EB];
+#pragma unroll
+        for (int j = 0; j < EB; ++j) {
+            const uint32_t k = base + j * BS + tid;
+            ok[j] = k < S;
+            uint32_t lo = 0, hi = BS;  // owner: the largest i with scan[i] <= k
+#pragma unroll
+            for (int step = 0; step < LOG_BS; ++step) {
+                uint32_t mid = (lo + hi) >> 1;
+                if (sm.scan[mid] <= k) lo = mid; else hi = mid;
+            }
+            uu[j] = sm.u[lo];
+            vv[j] = sm.uval[lo];
+            e[j] = sm.beg[lo] + (k - sm.scan[lo]);
         }
-    }
-    // big: CTA-cooperative
-    const uint32_t nb = sm.nbig;
-    for (uint32_t i = 0; i < nb; ++i) {
-        const uint32_t t = sm.big[i];
-        const uint32_t ub = sm.u[t], vb = sm.uval[t];
-        const Off bb = sm.beg[t];
-        const uint32_t db = sm.deg[t];
-        ops.edges_coop(ub, vb, bb, db, tid, BS);
+        ops.template batch<EB, true>(uu, vv, e, ok);
     }
     __syncthreads();
 }
@@ -436,7 +592,9 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, TileSmem<Off
         const Off b0 = a.rp[u], e0 = a.rp[u + 1];
         const Off b = b0 + (Off)k * HUB_CHUNK;
         const Off e = (e0 - b > (Off)HUB_CHUNK) ? b + HUB_CHUNK : e0;
-        ops.edges_coop(u, uval, b, (uint32_t)(e - b), threadIdx.x, BS);
+        constexpr uint32_t WIN = Ops<ALG, ORD, Off>::WIN;
+        const Off w0 = b / WIN, w1 = (e + WIN - 1) / WIN;
+        for (Off wi = w0 + (threadIdx.x >> 5); wi < w1; wi += WARPS_PER_CTA) ops.window(u, uval, wi * WIN, b, e);
     }
 }
 
@@ -472,11 +630,12 @@ __device__ __forceinline__ void compact_bitmap(const uint32_t *bm, uint32_t nwor
 // The persistent kernel
 // ------------------------------------------------------------------------------------------------
 template <int ALG, int ORD, typename Off>
-__global__ void __launch_bounds__(BS, MIN_BLOCKS) traverse_kernel(const TravArgs<Off> a) {
+__global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? AG_MINB_SSSP : AG_MINB_BFS)
+    traverse_kernel(const TravArgs<Off> a) {
     __shared__ TileSmem<Off> sm;
     Ctl *ctl = a.ctl;
     const uint32_t gtid = blockIdx.x * BS + threadIdx.x, gthreads = a.nblocks * BS;
-    const uint32_t src = a.src;
+    const uint32_t src = a.inv ? a.inv[a.src] : a.src;
     constexpr bool ROT = !(ALG == ALG_SSSP && ORD == ORD_O);
 
     // ---------------- phase 0: init (Fig. 4 lines 3-4; Fig. 8 lines 1-3) ----------------
@@ -490,13 +649,23 @@ __global__ void __launch_bounds__(BS, MIN_BLOCKS) traverse_kernel(const TravArgs
             a.P[v] = (v == src) ? (unsigned long long)src : INF64;   // dist 0, parent src
     }
     const uint32_t sbit = 1u << (src & 31), sword = src >> 5;
+#ifdef AG_EXPERIMENT   // ceiling experiments: one full sweep over every vertex (all already visited)
+    for (uint32_t wi = gtid; wi < a.nwords; wi += gthreads) {
+        const uint32_t full = (wi * 32 + 32 <= a.V) ? 0xFFFFFFFFu : ((1u << (a.V & 31)) - 1u);
+        a.bm[0][wi] = full;
+        a.bm[1][wi] = 0u;
+        a.bm[2][wi] = 0u;
+        if (ALG == ALG_BFS) a.vis[wi] = full;
+    }
+    if (false)
+#endif
     for (uint32_t wi = gtid; wi < a.nwords; wi += gthreads) {
         a.bm[0][wi] = (wi == sword) ? sbit : 0u;
         if (ROT) {
             a.bm[1][wi] = 0u;
             a.bm[2][wi] = 0u;
         }
-        if (ALG == ALG_BFS && ORD == ORD_O) a.vis[wi] = (wi == sword) ? sbit : 0u;
+        if (ALG == ALG_BFS) a.vis[wi] = (wi == sword) ? sbit : 0u;
     }
     if (gtid == 0) {
         a.q[0][0] = src;
@@ -508,7 +677,6 @@ __global__ void __launch_bounds__(BS, MIN_BLOCKS) traverse_kernel(const TravArgs
             ctl->hub_head[s] = 0;
             ctl->stage_done[s] = 0;
             ctl->it_edges[s] = 0;
-            ctl->it_verts[s] = 0;
         }
         ctl->pend_count = 1;
         ctl->overflow = 0;
@@ -518,6 +686,7 @@ __global__ void __launch_bounds__(BS, MIN_BLOCKS) traverse_kernel(const TravArgs
         ctl->eexp = 0;
     }
     grid_barrier(ctl, a.nblocks);
+    uint32_t n = 1;   // |WS_0| = |{src}|
 
     uint32_t prev_ws = WS_QU;   // representation used in the previous iteration
     uint8_t prev_var = 0;
@@ -525,46 +694,44 @@ __global__ void __launch_bounds__(BS, MIN_BLOCKS) traverse_kernel(const TravArgs
     uint32_t it = 0;
     for (;; ++it) {
         const uint32_t slot = it % 3;
-        const uint32_t n = ROT ? ld_relaxed(&ctl->q_len[slot]) : ld_relaxed(&ctl->pend_count);
         if (n == 0 || it >= a.max_iters) break;
         // decision maker, re-evaluated every sample_every iterations (inspector sampling, 26.s7-9)
         const uint8_t var = (it % a.pol.sample_every == 0 || prev_var == 0) ? select_variant(a.pol, n, 0) : prev_var;
         const uint32_t map = var >> 2, ws = var & 3;
         const uint32_t tag = a.epoch * 0x9E3779B1u + it + 1;
-
         if (blockIdx.x == 0 && threadIdx.x == 0) {
-            if (it > 0) {
-                const uint32_t ps = (it + 2) % 3;   // slot of iteration it-1
-                unsigned long long e = ctl->it_edges[ps], v = ctl->it_verts[ps];
-                ctl->eexp += e;
-                ctl->vexp += v;
-                if (it - 1 < a.trace_cap && a.trace_edges) a.trace_edges[it - 1] = e;
-            }
             if (it < a.trace_cap && a.trace_ws) {
                 a.trace_ws[it] = n;
                 a.trace_var[it] = var;
+                a.trace_ns[it] = globaltimer_ns();
+                if (it > 0) a.trace_edges[it - 1] = ld_relaxed64(&ctl->it_edges[(it + 2) % 3]);
             }
-            const uint32_t rs = (it + 2) % 3;       // reset slot(it+2) (last used by iteration it-1)
-            ctl->q_len[rs] = 0;
+            const uint32_t rs = (it + 2) % 3;   // reset slot(it+2): last used by iteration it-1,
+            ctl->q_len[rs] = 0;                 // next written in iteration it+1
             ctl->next_min[rs] = INF;
             ctl->tile_ctr[rs] = 0;
             ctl->hub_tail[rs] = 0;
             ctl->hub_head[rs] = 0;
             ctl->stage_done[rs] = 0;
             ctl->it_edges[rs] = 0;
-            ctl->it_verts[rs] = 0;
         }
 
         uint64_t hi = 0;
         bool append = true;
+        uint32_t qn = n;
         if (!ROT) {
             const uint32_t lo = ld_relaxed(&ctl->next_min[slot]);
             hi = (uint64_t)lo + a.pol.delta;
             append = (ws == WS_QU);
-            if (ws == WS_QU && prev_ws != WS_QU) {
-                // the pending list is stale: rebuild it from the pending bitmap
-                compact_bitmap(a.bm[0], a.nwords, a.q[slot], &ctl->q_len[slot], gtid >> 5, gthreads >> 5);
-                grid_barrier(ctl, a.nblocks);
+            if (ws == WS_QU) {
+                if (prev_ws != WS_QU) {
+                    // the pending list is stale: rebuild it from the pending bitmap
+                    compact_bitmap(a.bm[0], a.nwords, a.q[slot], &ctl->q_len[slot], gtid >> 5, gthreads >> 5);
+                    grid_barrier(ctl, a.nblocks);
+                    qn = ld_relaxed(&ctl->q_len[slot]);
+                } else {
+                    qn = ld_relaxed(&ctl->q_len[slot]);
+                }
             }
         } else {
             // clear the bitmap that iteration it+1 will write: bm[(it+2)%3] (read in iteration it-1)
@@ -580,56 +747,77 @@ __global__ void __launch_bounds__(BS, MIN_BLOCKS) traverse_kernel(const TravArgs
         }
 
         Ops<ALG, ORD, Off> ops(a, it, hi, append);
+        ops.wbuf = sm.wq[threadIdx.x >> 5];
         const uint32_t *bmc = ROT ? a.bm[slot] : a.bm[0];
         const uint32_t *qc = a.q[slot];
-        const uint32_t qn = ROT ? n : ld_relaxed(&ctl->q_len[slot]);
-        const uint32_t ntiles = (ws == WS_BM) ? (a.V + BS - 1) / BS : (qn + BS - 1) / BS;
+        // queue tiles: BS entries for thread mapping (element per thread); for the cooperative
+        // mappings a short queue is spread over all CTAs (>= 2 tiles per CTA)
+        uint32_t tile_n = BS;
+        if (ws == WS_QU && map != MAP_T) {
+            uint32_t want = (qn + 2 * a.nblocks - 1) / (2 * a.nblocks);
+            tile_n = want < 1u ? 1u : (want > (uint32_t)BS ? (uint32_t)BS : want);
+        }
+        // entry slot of this thread: spread across warps for the warp mapping
+        const uint32_t s_idx = (map == MAP_W || (map == MAP_B && a.pol.cta_group == 32))
+                                   ? (lane_id() * WARPS_PER_CTA + (threadIdx.x >> 5)) : threadIdx.x;
+        const uint32_t ntiles = (ws == WS_BM) ? (a.V + BS - 1) / BS : (qn + tile_n - 1) / tile_n;
         const bool hubs = (map == MAP_H) && a.has_hubs;
 
-        // dynamic tile scheduler: first tile static, then one atomic per tile
+        // dynamic tile scheduler: first tile static, then one atomic per tile, fetched one tile ahead
+        // (double-buffered in smem; the __syncthreads_or below orders the write before the read)
         uint32_t t = blockIdx.x;
+        int par = 0;
         while (t < ntiles) {
+            if (threadIdx.x == 0) sm.tnext[par] = a.nblocks + atomicAdd(&ctl->tile_ctr[slot], 1u);
             bool valid;
             uint32_t u;
             if (ws == WS_BM) {
                 u = t * BS + threadIdx.x;
                 valid = u < a.V && ((bmc[u >> 5] >> (u & 31)) & 1u);
             } else {
-                uint32_t i = t * BS + threadIdx.x;
-                valid = i < qn;
+                uint32_t i = t * tile_n + s_idx;
+                valid = s_idx < tile_n && i < qn;
                 u = valid ? qc[i] : 0u;
             }
-            process_tile(ops, sm, map, valid, u, a.pol.cta_group, hubs, slot, tag);
-            __syncthreads();
-            if (threadIdx.x == 0) sm.tile = a.nblocks + atomicAdd(&ctl->tile_ctr[slot], 1u);
-            __syncthreads();
-            t = sm.tile;
+            if (__syncthreads_or(valid))  // skip empty tiles (sparse bitmap): uniform branch
+                process_tile(ops, sm, map, valid, u, a.pol.cta_group, hubs, slot, tag);
+            t = sm.tnext[par];
+            par ^= 1;
         }
         if (hubs) drain_hubs(ops, sm, slot, tag);
+        ops.warp_flush(true);
         block_reduce_flush(ops, sm, ctl, slot);
         grid_barrier(ctl, a.nblocks);
+        n = ROT ? ld_relaxed(&ctl->q_len[(it + 1) % 3]) : ld_relaxed(&ctl->pend_count);
         prev_ws = ws;
         prev_var = var;
-        n_prev = n;
+        n_prev = qn;
     }
 
     // ---------------- termination ----------------
     if (blockIdx.x == 0 && threadIdx.x == 0) {
-        if (it > 0) {
-            const uint32_t ps = (it + 2) % 3;
-            unsigned long long e = ctl->it_edges[ps], v = ctl->it_verts[ps];
-            ctl->eexp += e;
-            ctl->vexp += v;
-            if (it - 1 < a.trace_cap && a.trace_edges) a.trace_edges[it - 1] = e;
-        }
         ctl->iterations = it;
+        if (it > 0 && it - 1 < a.trace_cap && a.trace_edges) a.trace_edges[it - 1] = ld_relaxed64(&ctl->it_edges[(it + 2) % 3]);
         if (it >= a.max_iters) ctl->aborted = 1;
+        if (it <= a.trace_cap && a.trace_ns) a.trace_ns[it] = globaltimer_ns();
     }
-    if (ALG == ALG_SSSP) {  // unpack (dist, parent) into the caller's arrays
+    if (ALG == ALG_SSSP) {  // unpack (dist, parent) into the caller's arrays (caller ids)
         for (uint32_t v = gtid; v < a.V; v += gthreads) {
-            unsigned long long pv = a.P[v];
+            unsigned long long pv = a.P[a.inv ? a.inv[v] : v];
             a.dist_out[v] = (uint32_t)(pv >> 32);
-            if (a.parent_out) a.parent_out[v] = (pv == INF64) ? INF : (uint32_t)pv;
+            if (a.parent_out) {
+                uint32_t pp = (uint32_t)pv;
+                a.parent_out[v] = (pv == INF64) ? INF : (a.perm ? a.perm[pp] : pp);
+            }
+        }
+    } else if (a.inv) {     // BFS in the degree layout: gather back to caller ids
+        for (uint32_t v = gtid; v < a.V; v += gthreads) {
+            const uint32_t i = a.inv[v];
+            a.out_level[v] = a.level[i];
+            if (a.out_parent) {
+                uint32_t pp = a.parent[i];
+                a.out_parent[v] = pp == INF ? INF : a.perm[pp];
+            }
         }
     }
 }

@@ -92,13 +92,15 @@ def check_sssp(g, G, s, p):
 
 
 # ------------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("layout", [0, 2])
 @pytest.mark.parametrize("seed", range(8))
-def test_tiny_random_all_variants(seed):
+def test_tiny_random_all_variants(seed, layout):
     rng = np.random.default_rng(seed)
     V = int(rng.integers(1, 300))
     g = aggen.random_graph(V, int(rng.integers(0, 6 * V + 1)), seed=seed, wmax=int(rng.integers(1, 100)),
                            sort_rows=bool(seed % 2))
-    G = A.Graph.from_csr(g)
+    G = A.Graph.from_csr(g, layout=layout)
+    assert G.info.layout in (1, 2) and (layout == 0 or G.info.layout == layout)
     srcs = sorted(set([0, V - 1, int(rng.integers(0, V))]))
     for p in all_policies():
         for s in srcs:
@@ -126,9 +128,10 @@ def test_c1_all_sources_adaptive():
             check_sssp(g, G, s, pol(0, kind=kind))
 
 
-def test_c1_all_static_variants():
+@pytest.mark.parametrize("layout", [1, 2])
+def test_c1_all_static_variants(layout):
     g = aggen.config("C1")
-    G = A.Graph.from_csr(g)
+    G = A.Graph.from_csr(g, layout=layout)
     for s in aggen.sources(g, 4, seed=11):
         for p in all_policies():
             check_bfs(g, G, s, p)
@@ -169,12 +172,13 @@ def test_closed_form_grid_and_path():
     assert np.array_equal(out, np.abs(np.arange(5000) - 17).astype(np.uint32)) and st.iterations == 4983
 
 
-def test_hubs_and_star():
+@pytest.mark.parametrize("layout", [1, 2])
+def test_hubs_and_star(layout):
     """Degree >> HUB_DEG exercises hub splitting (hybrid) and long CTA loops (paper variants)."""
     n = 300_000
     g = aggen.star(n)
     aggen.with_weights(g, seed=4, wmax=100)
-    G = A.Graph.from_csr(g)
+    G = A.Graph.from_csr(g, layout=layout)
     for p in [pol(0), pol(1), pol(0, 4, 2), pol(0, 4, 1), pol(0, 1, 2), pol(0, 3, 1), pol(1, 4, 2)]:
         for s in (0, 5):
             check_bfs(g, G, s, p)
@@ -254,6 +258,7 @@ def test_device_buffers_and_async():
 def test_full_size_configs(cfg):
     g = aggen.config(cfg)
     G = A.Graph.from_csr(g)
+    assert G.info.layout == (2 if cfg == "C2" else 1)   # inspector: skewed degrees -> degree layout
     srcs = [0] if cfg.startswith("C3") else []
     srcs += [int(s) for s in aggen.sources(g, 2)]
     for s in srcs:
