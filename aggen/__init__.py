@@ -61,6 +61,8 @@ def _L():
         _lib.aggen_sources.argtypes = [u32, ctypes.c_void_p, u64, u32, ctypes.c_void_p]
         _lib.aggen_free.argtypes = [ctypes.POINTER(_CSR)]
         _lib.aggen_free.restype = None
+        _lib.aggen_set_owned.argtypes = [u32, u32]
+        _lib.aggen_set_owned.restype = None
     return _lib
 
 
@@ -97,6 +99,16 @@ def rmat(scale: int, edgefactor: int = 16, seed: int = 1, a: float = 0.57, b: fl
     if rc != 0:
         raise RuntimeError(f"aggen_rmat failed ({rc})")
     return _take(cs, f"rmat{scale}_ef{edgefactor}_s{seed}")
+
+
+def rmat_part(scale: int, edgefactor: int, seed: int, own_b: int, own_e: int) -> Graph:
+    """The CSR entries of rmat(scale, edgefactor, seed) whose DESTINATION is in [own_b, own_e) (rows over
+    all V): exactly one rank's part of the 1-D destination partition, generated without the rest."""
+    _L().aggen_set_owned(own_b, own_e)
+    try:
+        return rmat(scale, edgefactor, seed)
+    finally:
+        _L().aggen_set_owned(0, 0xFFFFFFFF)
 
 
 def er(n: int, m: int, seed: int = 1) -> Graph:

@@ -151,6 +151,11 @@ static void sort_u32(uint32_t *a, uint64_t n, uint32_t *tmp) {
     free(cnt);
 }
 
+/* keep only CSR entries whose destination is in [own_b, own_e) (multi-GPU 1-D partition);
+ * own_b = 0, own_e = V keeps everything */
+static uint32_t g_own_b = 0, g_own_e = 0xFFFFFFFFu;
+static inline int owned(uint32_t v) { return v >= g_own_b && v < g_own_e; }
+
 static int build_csr(const gen_t *g, uint32_t V, uint64_t M, aggen_csr *out) {
     uint64_t *deg = (uint64_t *)calloc((size_t)V + 1, sizeof(uint64_t));
     if (!deg) return -1;
@@ -159,8 +164,8 @@ static int build_csr(const gen_t *g, uint32_t V, uint64_t M, aggen_csr *out) {
     for (int64_t i = 0; i < (int64_t)M; ++i) {
         uint32_t u, v;
         if (!gen_tuple(g, (uint64_t)i, &u, &v) || u == v) continue;
-        __atomic_fetch_add(&deg[u], 1, __ATOMIC_RELAXED);
-        __atomic_fetch_add(&deg[v], 1, __ATOMIC_RELAXED);
+        if (owned(v)) __atomic_fetch_add(&deg[u], 1, __ATOMIC_RELAXED);
+        if (owned(u)) __atomic_fetch_add(&deg[v], 1, __ATOMIC_RELAXED);
     }
     uint64_t *off = (uint64_t *)malloc(((size_t)V + 1) * sizeof(uint64_t));
     if (!off) { free(deg); return -1; }
@@ -176,10 +181,8 @@ static int build_csr(const gen_t *g, uint32_t V, uint64_t M, aggen_csr *out) {
     for (int64_t i = 0; i < (int64_t)M; ++i) {
         uint32_t u, v;
         if (!gen_tuple(g, (uint64_t)i, &u, &v) || u == v) continue;
-        uint64_t p = __atomic_fetch_add(&deg[u], 1, __ATOMIC_RELAXED);
-        col[p] = v;
-        p = __atomic_fetch_add(&deg[v], 1, __ATOMIC_RELAXED);
-        col[p] = u;
+        if (owned(v)) col[__atomic_fetch_add(&deg[u], 1, __ATOMIC_RELAXED)] = v;
+        if (owned(u)) col[__atomic_fetch_add(&deg[v], 1, __ATOMIC_RELAXED)] = u;
     }
     /* sort + dedup each row; deg[u] := unique count */
 #pragma omp parallel
@@ -302,3 +305,9 @@ void aggen_free(aggen_csr *g) {
 }
 
 int aggen_num_threads(void) { return omp_get_max_threads(); }
+
+/* restrict subsequent generators to destinations in [b, e) (call with 0, 0xFFFFFFFF to reset) */
+void aggen_set_owned(uint32_t b, uint32_t e) {
+    g_own_b = b;
+    g_own_e = e;
+}

@@ -8,8 +8,9 @@ adaptive (unordered) SSSP from source s_k of config C2 (R-MAT scale 22, edgefact
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl agraph|reference] [--config C2]
 
-N > 1 (torchrun): every rank runs independent queries (different sources) on its own GPU —
-independent problems, no data-path collective — "scaling": "weak".
+N > 1 (torchrun): config C5 — R-MAT scale 26 (AG_DIST_SCALE), BFS partitioned 1-D across the N GPUs by
+destination with one NCCL all-gather of the frontier bitmap per level; each rank
+generates only its own part.  "scaling": "strong" (fixed graph).
 --impl reference: the CPU oracle (serial queue BFS + heap Dijkstra, the paper's own baselines,
 PAPER.md:26.s21, 26.s36) timed on this host, rank 0 only.
 """
@@ -175,6 +176,73 @@ def cpu_baseline(g, srcs, budget_s=20.0):
             "sample": f"{n} sources x (queue BFS + heap Dijkstra) on the full graph, serial, {t:.1f}s"}
 
 
+def run_dist(args, rank, world, local, dist):
+    """C5: R-MAT scale 26 BFS partitioned across the ranks (strong scaling)."""
+    import torch
+    import aggen
+    from paper_conf_ipps_lib13_b200 import agraph as A
+    scale = int(os.environ.get("AG_DIST_SCALE", "26"))
+    V = 1 << scale
+    # NCCL bootstrap of the library's own communicator over the torch process group
+    uid = A.dist_unique_id() if rank == 0 else bytes(128)
+    t = torch.frombuffer(bytearray(uid), dtype=torch.uint8).clone().cuda()
+    dist.broadcast(t, 0)
+    comm = A.Comm.nccl(rank, world, bytes(t.cpu().numpy()), local)
+    b, e = A.owned_range(V, rank, world)
+    part = aggen.rmat_part(scale, 16, 1, b, e)
+    G = A.DistGraph(comm, V, part.row_ptr, part.col, local=True)
+    # sources with global degree >= 1 (local degrees summed over the ranks)
+    cand = np.unique((np.arange(256, dtype=np.uint64) * np.uint64(0x9E3779B97F4A7C15)) % np.uint64(V)).astype(np.int64)
+    ldeg = torch.from_numpy(np.diff(part.row_ptr)[cand].astype(np.int64)).cuda()
+    dist.all_reduce(ldeg)
+    srcs = cand[ldeg.cpu().numpy() > 0][:64]
+    lev = torch.empty(e - b, dtype=torch.int32, device="cuda")
+    stream = torch.cuda.current_stream()
+    for k in range(args.warmup):
+        G.bfs(int(srcs[k % len(srcs)]), levels=lev, stream=stream.cuda_stream)
+    K = args.steps
+    edges = 0
+    dist.barrier()
+    torch.cuda.synchronize()
+    sampler = ClockSampler(local)
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    l0 = A.kernel_launches()
+    with sampler:
+        start.record(stream)
+        for k in range(K):
+            _, _, st = G.bfs(int(srcs[k % len(srcs)]), levels=lev, stats=True, stream=stream.cuda_stream)
+            edges += st.edges_inspected
+        end.record(stream)
+        torch.cuda.synchronize()
+    dist.barrier()
+    t_ms = start.elapsed_time(end)
+    tt = torch.tensor([t_ms], device="cuda")
+    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    ee = torch.tensor([float(edges)], dtype=torch.float64, device="cuda")
+    dist.all_reduce(ee)          # sum of per-rank inspected edges = E_r per query (destination split)
+    t_ms, edges = float(tt.item()), float(ee.item())
+    peak, peak_src = measured_peak()
+    off = G.info.offset_bytes
+    # per-GPU compulsory bytes: its slice of the CSR + row offsets of the whole frontier + owned outputs
+    b_gpu = (edges / K / world) * 4 + V * (2 * off) + (e - b) * 8
+    achieved = b_gpu / (t_ms / K * 1e-3) / 1e9
+    out = {"metric": "BFS/SSSP GTEPS (device-timed); fraction of HBM roofline", "value": edges / (t_ms * 1e-3) / 1e9,
+           "unit": "GTEPS", "n_gpus": world, "steps": K, "warmup": args.warmup, "ms_per_step": t_ms / K,
+           "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+           "config": {"workload": f"C5: R-MAT scale-{scale} ef16 BFS, 1-D destination partition over {world} GPUs, "
+                                  f"per-level NCCL all-gather of the frontier bitmap", "V": V,
+                      "parallelism": f"1-D partition x{world}", "l2": "inputs larger than L2"},
+           "roofline": {"bound": "hbm", "kernel": "dist_level_kernel", "achieved": achieved, "peak": peak,
+                        "peak_source": peak_src, "unit": "GB/s", "frac": achieved / peak, "traffic": None},
+           "gpu_launches": A.kernel_launches() - l0, "clocks": sampler.summary(),
+           "e2e": {"value": None, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
+                   "note": "multi-GPU e2e not measured this round"}}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    G.free()
+    comm.free()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -199,12 +267,17 @@ def main():
     from paper_conf_ipps_lib13_b200 import agraph as A
     from paper_conf_ipps_lib13_b200 import build as B
 
-    B.build()
+    if rank == 0:
+        B.build()
     torch.cuda.set_device(local)
     dist = None
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        dist.barrier()
+        run_dist(args, rank, world, local, dist)
+        dist.destroy_process_group()
+        return
 
     g = aggen.config(args.config)
     G = A.Graph.from_csr(g, device=local)

@@ -204,6 +204,19 @@ ag_status ag_dist_owned_range(uint32_t V, int rank, int world, uint32_t *begin, 
 /* Every rank passes the SAME global CSR (host or device); each keeps its destination-owned part. */
 ag_status ag_dist_graph_load_csr(ag_comm c, uint32_t V, uint64_t E, const uint64_t *row_ptr,
                                  const uint32_t *col_idx, const uint32_t *weights, ag_graph *out_local);
+/* As above but every rank passes only ITS part: CSR rows over all V whose entries all have their
+ * destination in the rank's owned range (AG_ERR_BAD_CSR otherwise).  Lets each process build its
+ * part without holding the whole graph (R-MAT scale 26 = 8.6 GB of col_idx). */
+ag_status ag_dist_graph_load_local(ag_comm c, uint32_t V, uint64_t E_local, const uint64_t *row_ptr,
+                                   const uint32_t *col_idx, const uint32_t *weights, ag_graph *out_local);
+/* Virtual group for tests on ONE GPU: creates `world` comms (ranks 0..world-1) in this process on
+ * `device`; their all-gather is a device copy.  Load each rank's part with ag_dist_graph_load_csr
+ * and run them in lock step with ag_dist_bfs_group.  comms_out: array of `world` handles. */
+ag_status ag_dist_init_local(int world, int device, ag_comm *comms_out);
+/* Lock-step BFS over all ranks of a virtual group (locals[r] = rank r's part); levels_owned[r] /
+ * parents_owned[r] (nullable) receive rank r's owned slices. */
+ag_status ag_dist_bfs_group(ag_graph *locals, int world, uint32_t src, uint32_t **levels_owned,
+                            uint32_t **parents_owned, ag_run_stats *stats, void *stream);
 /* Distributed BFS (unordered = ordered level-synchronous here).  levels_owned / parents_owned:
  * (end - begin) uint32 for this rank's owned range.  Collective: all ranks call with the same src. */
 ag_status ag_dist_bfs(ag_graph local, uint32_t src, uint32_t *levels_owned, uint32_t *parents_owned,

@@ -69,10 +69,11 @@ class RunStats(ctypes.Structure):
                 ("trace_variant", ctypes.POINTER(ctypes.c_uint8)), ("trace_ns", ctypes.POINTER(ctypes.c_uint64))]
 
 
-EXPORTS = ["ag_policy_default", "ag_select", "ag_graph_load_csr", "ag_graph_load_csr_ex", "ag_graph_info_get", "ag_graph_free", "ag_bfs",
-           "ag_sssp", "ag_graph_check", "ag_dist_unique_id", "ag_dist_init", "ag_dist_free", "ag_dist_owned_range",
-           "ag_dist_graph_load_csr", "ag_dist_bfs", "ag_set_allocator", "ag_status_string", "ag_last_error",
-           "ag_abi_version", "ag_kernel_launches"]
+EXPORTS = ["ag_policy_default", "ag_select", "ag_graph_load_csr", "ag_graph_load_csr_ex", "ag_graph_info_get",
+           "ag_graph_free", "ag_bfs", "ag_sssp", "ag_graph_check", "ag_dist_unique_id", "ag_dist_init",
+           "ag_dist_init_local", "ag_dist_free", "ag_dist_owned_range", "ag_dist_graph_load_csr",
+           "ag_dist_graph_load_local", "ag_dist_bfs", "ag_dist_bfs_group", "ag_set_allocator", "ag_status_string",
+           "ag_last_error", "ag_abi_version", "ag_kernel_launches"]
 
 _lib = None
 
@@ -84,6 +85,14 @@ def lib():
         return _lib
     if not os.path.exists(LIB_PATH):
         raise AgError(10, f"{LIB_PATH} not built; run python -m paper_conf_ipps_lib13_b200.build")
+    if "AG_NCCL_LIB" not in os.environ:  # the library dlopens NCCL on first multi-GPU use
+        try:
+            import nvidia.nccl as _n
+            cand = os.path.join(list(_n.__path__)[0], "lib", "libnccl.so.2")
+            if os.path.exists(cand):
+                os.environ["AG_NCCL_LIB"] = cand
+        except Exception:
+            pass
     L = ctypes.CDLL(LIB_PATH)
     vp, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
     L.ag_policy_default.argtypes = [ctypes.POINTER(Policy), i32]
@@ -102,6 +111,9 @@ def lib():
     L.ag_dist_owned_range.argtypes = [u32, i32, i32, ctypes.POINTER(u32), ctypes.POINTER(u32)]
     L.ag_dist_graph_load_csr.argtypes = [vp, u32, u64, vp, vp, vp, ctypes.POINTER(vp)]
     L.ag_dist_bfs.argtypes = [vp, u32, vp, vp, ctypes.POINTER(Policy), ctypes.POINTER(RunStats), vp]
+    L.ag_dist_init_local.argtypes = [i32, i32, vp]
+    L.ag_dist_graph_load_local.argtypes = [vp, u32, u64, vp, vp, vp, ctypes.POINTER(vp)]
+    L.ag_dist_bfs_group.argtypes = [vp, i32, u32, vp, vp, ctypes.POINTER(RunStats), vp]
     L.ag_status_string.restype = ctypes.c_char_p
     L.ag_status_string.argtypes = [i32]
     L.ag_last_error.restype = ctypes.c_char_p
@@ -228,3 +240,107 @@ class Graph:
 
     def check(self):
         _check(lib().ag_graph_check(self.h))
+
+
+# ---------------------------------------------------------------------------------------------
+# multi-GPU (1-D destination partition)
+# ---------------------------------------------------------------------------------------------
+def owned_range(V: int, rank: int, world: int):
+    b, e = ctypes.c_uint32(), ctypes.c_uint32()
+    _check(lib().ag_dist_owned_range(V, rank, world, ctypes.byref(b), ctypes.byref(e)))
+    return b.value, e.value
+
+
+def dist_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().ag_dist_unique_id(buf))
+    return buf.raw
+
+
+class Comm:
+    """One rank's communicator: NCCL (ag_dist_init) or a member of a virtual group."""
+
+    def __init__(self, handle, rank: int, world: int, device: int):
+        self.h, self.rank, self.world, self.device = handle, rank, world, device
+
+    @classmethod
+    def nccl(cls, rank: int, world: int, unique_id: bytes, device: int):
+        h = ctypes.c_void_p()
+        idbuf = ctypes.create_string_buffer(unique_id, 128)
+        _check(lib().ag_dist_init(rank, world, idbuf, device, ctypes.byref(h)))
+        return cls(h, rank, world, device)
+
+    def free(self):
+        if self.h:
+            _check(lib().ag_dist_free(self.h))
+            self.h = None
+
+
+def local_group(world: int, device: int = 0):
+    """`world` virtual ranks in this process on one GPU (all-gather = device copy)."""
+    arr = (ctypes.c_void_p * world)()
+    _check(lib().ag_dist_init_local(world, device, arr))
+    return [Comm(ctypes.c_void_p(arr[r]), r, world, device) for r in range(world)]
+
+
+class DistGraph(Graph):
+    """This rank's part of a 1-D destination-partitioned graph."""
+
+    def __init__(self, comm: Comm, V: int, row_ptr, col, w=None, local: bool = False):
+        h = ctypes.c_void_p()
+        E = int(row_ptr[-1]) if isinstance(row_ptr, np.ndarray) else int(row_ptr[-1].item())
+        fn = lib().ag_dist_graph_load_local if local else lib().ag_dist_graph_load_csr
+        _check(fn(comm.h, V, E, _ptr(row_ptr), _ptr(col), _ptr(w), ctypes.byref(h)))
+        self.h, self.V, self.E, self.device, self.comm = h, V, E, comm.device, comm
+        self.own = owned_range(V, comm.rank, comm.world)
+        self.info = GraphInfo()
+        _check(lib().ag_graph_info_get(self.h, ctypes.byref(self.info)))
+
+    def bfs(self, src: int, levels=None, parents=None, policy=None, stats: bool = False, trace_cap: int = 0,
+            stream=None):
+        """ag_dist_bfs (collective over the NCCL communicator): returns this rank's owned slices."""
+        n = self.own[1] - self.own[0]
+        if levels is None:
+            levels = np.empty(n, np.uint32)
+        st, tr = _mkstats(stats, trace_cap)
+        _check(lib().ag_dist_bfs(self.h, int(src), _ptr(levels), _ptr(parents),
+                                 ctypes.byref(policy) if policy is not None else None,
+                                 ctypes.byref(st) if st is not None else None, ctypes.c_void_p(stream or 0)))
+        return levels, parents, _stats_out(st, tr)
+
+
+def dist_bfs_group(parts, src: int, parents: bool = False, stats: bool = False, trace_cap: int = 0):
+    """Lock-step BFS over the ranks of a virtual group; returns (levels, parents|None, Stats) in
+    GLOBAL vertex order (owned slices concatenated)."""
+    P = len(parts)
+    lv = [np.empty(p.own[1] - p.own[0], np.uint32) for p in parts]
+    pa = [np.empty(p.own[1] - p.own[0], np.uint32) for p in parts] if parents else None
+    hs = (ctypes.c_void_p * P)(*[p.h.value for p in parts])
+    lvp = (ctypes.c_void_p * P)(*[a.ctypes.data for a in lv])
+    pap = (ctypes.c_void_p * P)(*[a.ctypes.data for a in pa]) if parents else None
+    st, tr = _mkstats(stats, trace_cap)
+    _check(lib().ag_dist_bfs_group(hs, P, int(src), lvp, pap, ctypes.byref(st) if st is not None else None, None))
+    return np.concatenate(lv), (np.concatenate(pa) if parents else None), _stats_out(st, tr)
+
+
+def _mkstats(stats, trace_cap):
+    if not stats:
+        return None, None
+    st = RunStats()
+    st.struct_size = ctypes.sizeof(RunStats)
+    tr = None
+    if trace_cap:
+        tr = (np.zeros(trace_cap, np.uint32), np.zeros(trace_cap, np.uint64), np.zeros(trace_cap, np.uint8),
+              np.zeros(trace_cap + 1, np.uint64))
+        st.trace_cap = trace_cap
+        st.trace_ws = tr[0].ctypes.data_as(ctypes.POINTER(ctypes.c_uint32))
+    return st, tr
+
+
+def _stats_out(st, tr):
+    if st is None:
+        return None
+    res = Stats(st.iterations, st.vertices_expanded, st.edges_inspected, st.reached, st.reached_edges, st.device_ms)
+    if tr is not None:
+        res.trace_ws = tr[0][: st.trace_len]
+    return res

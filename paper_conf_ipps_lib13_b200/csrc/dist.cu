@@ -1,12 +1,314 @@
-// dist.cu — multi-GPU 1-D destination partition.  Placeholder entry points until the
-// NCCL path lands; every call reports AG_ERR_UNSUPPORTED.
+// dist.cu — multi-GPU BFS: 1-D destination partition, per-level frontier-bitmap all-gather.
+//
+// Not in the paper (one C2070, PAPER.md:26.s15); required by BASELINE.json north_star / SURVEY.md §8(e).
+//  * Rank p owns vertices [p*S, min(V,(p+1)*S)), S = ceil(V/P) rounded up to 1024 (whole 128-B bitmap
+//    slices).  It stores every CSR entry whose DESTINATION it owns, indexed by source over all V, so
+//    expanding any frontier vertex touches only owned level/visited entries: no remote writes, no
+//    cross-GPU atomics (NCCL has no bitwise-OR reduction; destination ownership needs none).
+//  * Per level: the identical global frontier bitmap (V/8 B) is compacted to a local queue
+//    (O(V/32) warp scan), expanded over the local CSR with the load-balanced hybrid mapping
+//    (a4), the owned next-frontier slice is published with ncclAllGather(slice -> global bitmap)
+//    over NVLink, and termination is a popcount of the gathered bitmap on every rank (no extra
+//    collective).
+//  * Transport: NCCL (one process per GPU), or a "local group" of P virtual ranks inside one
+//    process on one GPU whose all-gather is a device copy — used by the tests to check the
+//    partitioning / ownership logic at any P on a single device.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <vector>
+
+#include <cub/device/device_scan.cuh>
+
 #include "agraph.h"
+#include "common.cuh"
 #include "graph.h"
+#include "traverse.cuh"
+
+// Minimal NCCL ABI declarations (nccl.h 2.x): the library dlopens libnccl.so.2 at run time.
+typedef struct ncclComm *ncclComm_t;
+typedef struct { char internal[128]; } ncclUniqueId;
+typedef enum { ncclSuccess = 0 } ncclResult_t;
+typedef enum { ncclUint8 = 1 } ncclDataType_t;
+
+namespace {
+
+// ---- NCCL loaded at run time (the library itself must load without NCCL)
+struct NcclApi {
+    bool ok = false;
+    ncclResult_t (*GetUniqueId)(ncclUniqueId *) = nullptr;
+    ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*AllGather)(const void *, void *, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+    const char *(*GetErrorString)(ncclResult_t) = nullptr;
+};
+NcclApi g_nccl;
+std::mutex g_nccl_mu;
+
+bool load_nccl() {
+    std::lock_guard<std::mutex> lk(g_nccl_mu);
+    if (g_nccl.ok) return true;
+    void *h = nullptr;
+    if (const char *p = getenv("AG_NCCL_LIB")) h = dlopen(p, RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return false;
+    g_nccl.GetUniqueId = (decltype(g_nccl.GetUniqueId))dlsym(h, "ncclGetUniqueId");
+    g_nccl.CommInitRank = (decltype(g_nccl.CommInitRank))dlsym(h, "ncclCommInitRank");
+    g_nccl.CommDestroy = (decltype(g_nccl.CommDestroy))dlsym(h, "ncclCommDestroy");
+    g_nccl.AllGather = (decltype(g_nccl.AllGather))dlsym(h, "ncclAllGather");
+    g_nccl.GetErrorString = (decltype(g_nccl.GetErrorString))dlsym(h, "ncclGetErrorString");
+    g_nccl.ok = g_nccl.GetUniqueId && g_nccl.CommInitRank && g_nccl.CommDestroy && g_nccl.AllGather;
+    return g_nccl.ok;
+}
+
+ag_status nccl_status(ncclResult_t r, const char *what) {
+    if (r == ncclSuccess) return AG_OK;
+    return ag::set_error(AG_ERR_NCCL, "%s: %s", what, g_nccl.GetErrorString ? g_nccl.GetErrorString(r) : "nccl error");
+}
+
+}  // namespace
+
+struct ag_local_group;
+
+struct ag_comm_s {
+    int rank = 0, world = 1, device = 0;
+    ncclComm_t nccl = nullptr;
+    ag_local_group *group = nullptr;   // virtual mode
+};
+
+struct ag_local_group {
+    int world = 0;
+    int refs = 0;                      // live comms of the group
+    std::vector<ag_graph_s *> parts;   // registered local graphs, index = rank
+};
+
+struct ag_dist_part {
+    ag_comm_s *comm = nullptr;
+    uint32_t own_b = 0, own_e = 0;     // owned vertex range
+    uint32_t S = 0;                    // slice size (bits), multiple of 1024
+    uint32_t gwords = 0;               // words of the padded global bitmap (world * S / 32)
+    uint32_t *d_front = nullptr;       // global frontier bitmap (gathered)
+    uint32_t *d_next = nullptr;        // next-frontier bitmap (only owned words written)
+    unsigned long long *d_cnt = nullptr;
+    unsigned long long *h_cnt = nullptr;  // pinned
+};
 
 namespace ag {
-void dist_graph_release(ag_graph_s *) {}
+
+void dist_graph_release(ag_graph_s *g) {
+    if (!g->dist) return;
+    ag_dist_part *d = g->dist;
+    dev_free(d->d_front, (size_t)d->gwords * 4 + 128, g->device);
+    dev_free(d->d_next, (size_t)d->gwords * 4 + 128, g->device);
+    dev_free(d->d_cnt, 64, g->device);
+    if (d->h_cnt) cudaFreeHost(d->h_cnt);
+    delete d;
+    g->dist = nullptr;
+}
+
 }  // namespace ag
 
+using namespace ag;
+
+// ------------------------------------------------------------------------------------------------
+// kernels
+// ------------------------------------------------------------------------------------------------
+// count the owned entries of each row
+__global__ void dist_count_kernel(const uint64_t *rp, const uint32_t *col, uint32_t V, uint32_t b, uint32_t e,
+                                  uint64_t *cnt) {
+    const uint32_t lane = threadIdx.x & 31, warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t u = warp; u < V; u += nwarps) {
+        uint64_t c = 0;
+        for (uint64_t k = rp[u] + lane; k < rp[u + 1]; k += 32) {
+            uint32_t v = col[k];
+            c += (v >= b && v < e);
+        }
+        c = warp_sum(c);
+        if (lane == 0) cnt[u] = c;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) cnt[V] = 0;
+}
+
+// scatter the owned entries (order within a row preserved by a warp ballot scan)
+__global__ void dist_scatter_kernel(const uint64_t *rp, const uint32_t *col, const uint32_t *w, uint32_t V,
+                                    uint32_t b, uint32_t e, const uint64_t *nrp, uint32_t *ncol, uint32_t *nw) {
+    const uint32_t lane = threadIdx.x & 31, warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t u = warp; u < V; u += nwarps) {
+        uint64_t out = nrp[u];
+        for (uint64_t k0 = rp[u]; k0 < rp[u + 1]; k0 += 32) {
+            const uint64_t k = k0 + lane;
+            uint32_t v = 0;
+            bool keep = false;
+            if (k < rp[u + 1]) {
+                v = col[k];
+                keep = v >= b && v < e;
+            }
+            const unsigned m = __ballot_sync(0xffffffffu, keep);
+            if (keep) {
+                const uint64_t pos = out + __popc(m & ((1u << lane) - 1u));
+                ncol[pos] = v;
+                if (w) nw[pos] = w[k];
+            }
+            out += __popc(m);
+        }
+    }
+}
+
+__global__ void dist_init_kernel(uint32_t *level, uint32_t *parent, uint32_t *vis, uint32_t *front, uint32_t *next,
+                                 uint32_t V, uint32_t gwords, uint32_t src) {
+    const uint32_t gt = blockIdx.x * blockDim.x + threadIdx.x, gs = gridDim.x * blockDim.x;
+    for (uint32_t v = gt; v < V; v += gs) {
+        level[v] = v == src ? 0u : INF;
+        if (parent) parent[v] = v == src ? src : INF;
+    }
+    for (uint32_t wi = gt; wi < gwords; wi += gs) {
+        const uint32_t bit = (wi == (src >> 5)) ? (1u << (src & 31)) : 0u;
+        vis[wi] = bit;
+        front[wi] = bit;
+        next[wi] = 0u;
+    }
+}
+
+__global__ void owned_check_kernel(const uint32_t *col, uint64_t E, uint32_t b, uint32_t e, unsigned *bad) {
+    for (uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < E; k += (uint64_t)gridDim.x * blockDim.x)
+        if (col[k] < b || col[k] >= e) *bad = 1;
+}
+
+__global__ void popcount_kernel(const uint32_t *bm, uint32_t nwords, unsigned long long *cnt) {
+    unsigned long long c = 0;
+    for (uint32_t wi = blockIdx.x * blockDim.x + threadIdx.x; wi < nwords; wi += gridDim.x * blockDim.x)
+        c += __popc(bm[wi]);
+    c = warp_sum(c);
+    if ((threadIdx.x & 31) == 0 && c) atomicAdd(cnt, c);
+}
+
+// One BFS level on one rank: compact the global frontier bitmap into a local queue (O(V/32)), grid
+// barrier, then expand it over the local (destination-owned) CSR with the hybrid mapping.  Discovered
+// owned vertices get their level and their bit in the next-frontier bitmap.
+template <typename Off>
+__global__ void __launch_bounds__(BS, AG_MINB_BFS) dist_level_kernel(const TravArgs<Off> a, uint32_t L,
+                                                                     const uint32_t *front) {
+    __shared__ TileSmem<Off> sm;
+    Ctl *ctl = a.ctl;
+    const uint32_t slot = 0;
+    const uint32_t gtid = blockIdx.x * BS + threadIdx.x, gthreads = a.nblocks * BS;
+    compact_bitmap(front, a.nwords, a.q[0], &ctl->q_len[0], gtid >> 5, gthreads >> 5);
+    grid_barrier(ctl, a.nblocks);
+    const uint32_t qn = ld_relaxed(&ctl->q_len[0]);
+    Ops<ALG_BFS, ORD_O, Off> ops(a, L, 0, true);
+    ops.wbuf = sm.wq[threadIdx.x >> 5];
+    uint32_t tile_n = (qn + 2 * a.nblocks - 1) / (2 * a.nblocks);
+    tile_n = tile_n < 1u ? 1u : (tile_n > (uint32_t)BS ? (uint32_t)BS : tile_n);
+    const uint32_t ntiles = (qn + tile_n - 1) / tile_n;
+    const uint32_t tag = a.epoch * 0x9E3779B1u + L + 1;
+    uint32_t t = blockIdx.x;
+    int par = 0;
+    while (t < ntiles) {
+        if (threadIdx.x == 0) sm.tnext[par] = a.nblocks + atomicAdd(&ctl->tile_ctr[slot], 1u);
+        const uint32_t i = t * tile_n + threadIdx.x;
+        const bool valid = threadIdx.x < tile_n && i < qn;
+        const uint32_t u = valid ? a.q[0][i] : 0u;
+        if (__syncthreads_or(valid)) process_tile(ops, sm, MAP_H, valid, u, 32u, a.has_hubs != 0, slot, tag);
+        t = sm.tnext[par];
+        par ^= 1;
+    }
+    if (a.has_hubs) drain_hubs(ops, sm, slot, tag);
+    ops.warp_flush(true);
+    block_reduce_flush(ops, sm, ctl, slot);
+}
+
+// ------------------------------------------------------------------------------------------------
+// host side
+// ------------------------------------------------------------------------------------------------
+namespace {
+
+ag_status part_alloc(ag_graph_s *g, ag_comm_s *c) {
+    ag_dist_part *d = new ag_dist_part();
+    d->comm = c;
+    ag_dist_owned_range(g->V, c->rank, c->world, &d->own_b, &d->own_e);
+    uint64_t S = ((uint64_t)g->V + c->world - 1) / c->world;
+    S = (S + 1023) & ~1023ull;
+    d->S = (uint32_t)S;
+    d->gwords = (uint32_t)(S * c->world / 32);
+    g->dist = d;
+    ag_status s;
+    if ((s = dev_alloc((void **)&d->d_front, (size_t)d->gwords * 4 + 128, g->device)) != AG_OK) return s;
+    if ((s = dev_alloc((void **)&d->d_next, (size_t)d->gwords * 4 + 128, g->device)) != AG_OK) return s;
+    if ((s = dev_alloc((void **)&d->d_cnt, 64, g->device)) != AG_OK) return s;
+    if (cudaMallocHost(&d->h_cnt, 64) != cudaSuccess) return set_error(AG_ERR_OOM, "pinned alloc");
+    return AG_OK;
+}
+
+// scratch the level kernel needs (same layout as the single-GPU handle; bitmaps sized to gwords)
+ag_status dist_scratch(ag_graph_s *g) {
+    ag_status s;
+    const size_t V = g->V, gw = g->dist->gwords;
+    if (!g->d_ctl) {
+        if ((s = dev_alloc(&g->d_ctl, sizeof(Ctl), g->device)) != AG_OK) return s;
+        cudaMemset(g->d_ctl, 0, sizeof(Ctl));
+        g->ctl_init = true;
+    }
+    if (!g->d_q[0] && (s = dev_alloc((void **)&g->d_q[0], V * 4 + 128, g->device)) != AG_OK) return s;
+    if (!g->d_q[1] && (s = dev_alloc((void **)&g->d_q[1], V * 4 + 128, g->device)) != AG_OK) return s;
+    if (!g->d_vis && (s = dev_alloc((void **)&g->d_vis, gw * 4 + 128, g->device)) != AG_OK) return s;
+    if (!g->d_hub && (s = dev_alloc((void **)&g->d_hub, (size_t)g->hub_cap * 16, g->device)) != AG_OK) return s;
+    if (!g->d_level && (s = dev_alloc((void **)&g->d_level, V * 4 + 128, g->device)) != AG_OK) return s;
+    if (!g->d_acc && (s = dev_alloc(&g->d_acc, 64, g->device)) != AG_OK) return s;
+    return AG_OK;
+}
+
+struct LevelCfg {
+    int nblocks = 0;
+};
+
+template <typename Off>
+ag_status launch_level(ag_graph_s *g, uint32_t L, uint32_t *parent_local, cudaStream_t st) {
+    ag_dist_part *d = g->dist;
+    TravArgs<Off> a;
+    memset(&a, 0, sizeof a);
+    a.rp = (const Off *)g->d_rp;
+    a.col = g->d_col;
+    a.V = g->V;
+    a.nwords = d->gwords;
+    a.level = g->d_level;
+    a.parent = parent_local;
+    a.vis = g->d_vis;
+    a.bm[0] = a.bm[1] = a.bm[2] = d->d_next;
+    a.q[0] = g->d_q[0];
+    a.q[1] = a.q[2] = g->d_q[1];   // appends of the expansion (not consumed: the bitmap is exchanged)
+    a.hub = g->d_hub;
+    a.hub_cap = g->hub_cap;
+    a.ctl = (Ctl *)g->d_ctl;
+    a.epoch = ++g->epoch;
+    a.has_hubs = g->info.max_deg >= HUB_DEG;
+    auto fn = dist_level_kernel<Off>;
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, BS, 0);
+    if (occ < 1) return set_error(AG_ERR_CUDA, "dist kernel does not fit");
+    a.nblocks = (uint32_t)(occ * g->num_sms);
+    // reset the per-level counters of slot 0/1 (q_len, tile/hub scheduler)
+    cudaMemsetAsync((char *)g->d_ctl + offsetof(Ctl, q_len), 0, offsetof(Ctl, it_edges) - offsetof(Ctl, q_len), st);
+    void *args[] = {(void *)&a, (void *)&L, (void *)&d->d_front};
+    cudaError_t e = cudaLaunchCooperativeKernel((const void *)fn, dim3(a.nblocks), dim3(BS), args, 0, st);
+    note_launch(1);
+    return cuda_status(e, "dist level");
+}
+
+ag_status run_level(ag_graph_s *g, uint32_t L, uint32_t *parent_local, cudaStream_t st) {
+    return g->offs32 ? launch_level<uint32_t>(g, L, parent_local, st)
+                     : launch_level<unsigned long long>(g, L, parent_local, st);
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------------------------------------
+// C ABI
+// ------------------------------------------------------------------------------------------------
 extern "C" {
 
 ag_status ag_dist_owned_range(uint32_t V, int rank, int world, uint32_t *begin, uint32_t *end) {
@@ -22,17 +324,296 @@ ag_status ag_dist_owned_range(uint32_t V, int rank, int world, uint32_t *begin, 
     return AG_OK;
 }
 
-ag_status ag_dist_unique_id(void *) { return ag::set_error(AG_ERR_UNSUPPORTED, "multi-GPU path not built yet"); }
-ag_status ag_dist_init(int, int, const void *, int, ag_comm *) {
-    return ag::set_error(AG_ERR_UNSUPPORTED, "multi-GPU path not built yet");
+ag_status ag_dist_unique_id(void *out128) {
+    if (!out128) return set_error(AG_ERR_INVALID_ARG, "NULL");
+    if (!load_nccl()) return set_error(AG_ERR_NCCL, "cannot load libnccl.so.2 (set AG_NCCL_LIB)");
+    ncclUniqueId id;
+    ag_status s = nccl_status(g_nccl.GetUniqueId(&id), "ncclGetUniqueId");
+    if (s == AG_OK) memcpy(out128, &id, sizeof id);
+    return s;
 }
-ag_status ag_dist_free(ag_comm) { return ag::set_error(AG_ERR_UNSUPPORTED, "multi-GPU path not built yet"); }
-ag_status ag_dist_graph_load_csr(ag_comm, uint32_t, uint64_t, const uint64_t *, const uint32_t *, const uint32_t *,
-                                 ag_graph *) {
-    return ag::set_error(AG_ERR_UNSUPPORTED, "multi-GPU path not built yet");
+
+ag_status ag_dist_init(int rank, int world, const void *id128, int device, ag_comm *out) {
+    if (!out || !id128 || world < 1 || rank < 0 || rank >= world) return set_error(AG_ERR_INVALID_ARG, "bad args");
+    ag_status s = check_device(device, nullptr);
+    if (s != AG_OK) return s;
+    if (!load_nccl()) return set_error(AG_ERR_NCCL, "cannot load libnccl.so.2 (set AG_NCCL_LIB)");
+    cudaSetDevice(device);
+    ncclUniqueId id;
+    memcpy(&id, id128, sizeof id);
+    ag_comm_s *c = new ag_comm_s();
+    c->rank = rank;
+    c->world = world;
+    c->device = device;
+    s = nccl_status(g_nccl.CommInitRank(&c->nccl, world, id, rank), "ncclCommInitRank");
+    if (s != AG_OK) {
+        delete c;
+        return s;
+    }
+    *out = c;
+    return AG_OK;
 }
-ag_status ag_dist_bfs(ag_graph, uint32_t, uint32_t *, uint32_t *, const ag_policy *, ag_run_stats *, void *) {
-    return ag::set_error(AG_ERR_UNSUPPORTED, "multi-GPU path not built yet");
+
+ag_status ag_dist_init_local(int world, int device, ag_comm *comms_out) {
+    if (!comms_out || world < 1) return set_error(AG_ERR_INVALID_ARG, "bad args");
+    ag_status s = check_device(device, nullptr);
+    if (s != AG_OK) return s;
+    ag_local_group *grp = new ag_local_group();
+    grp->world = world;
+    grp->refs = world;
+    grp->parts.assign(world, nullptr);
+    for (int r = 0; r < world; ++r) {
+        ag_comm_s *c = new ag_comm_s();
+        c->rank = r;
+        c->world = world;
+        c->device = device;
+        c->group = grp;
+        comms_out[r] = c;
+    }
+    return AG_OK;
+}
+
+ag_status ag_dist_free(ag_comm c) {
+    if (!c) return set_error(AG_ERR_INVALID_ARG, "NULL");
+    if (c->nccl && g_nccl.ok) g_nccl.CommDestroy(c->nccl);
+    if (c->group) {
+        c->group->parts[c->rank] = nullptr;
+        if (--c->group->refs == 0) delete c->group;
+    }
+    delete c;
+    return AG_OK;
+}
+
+ag_status ag_dist_graph_load_csr(ag_comm c, uint32_t V, uint64_t E, const uint64_t *row_ptr, const uint32_t *col_idx,
+                                 const uint32_t *weights, ag_graph *out_local) {
+    if (!c || !out_local || !row_ptr || (!col_idx && E)) return set_error(AG_ERR_INVALID_ARG, "NULL argument");
+    *out_local = nullptr;
+    if (V == 0 || V >= 0xFFFFFFFFu) return set_error(AG_ERR_BAD_CSR, "V must be in [1, 2^32-1)");
+    const int dev = c->device;
+    cudaSetDevice(dev);
+    uint32_t b, e;
+    ag_dist_owned_range(V, c->rank, c->world, &b, &e);
+    // validate the global CSR by loading it (identity layout), then extract the owned part
+    ag_graph g0 = nullptr;
+    ag_status s = ag_graph_load_csr_ex(V, E, row_ptr, col_idx, weights, dev, AG_LAYOUT_IDENTITY, &g0);
+    if (s != AG_OK) return s;
+    // global row offsets as u64 (the store may have narrowed them)
+    uint64_t *rp64 = nullptr, *cnt = nullptr, *nrp = nullptr;
+    uint32_t *ncol = nullptr, *nw = nullptr;
+    const int grid = g0->num_sms * 8;
+    if ((s = dev_alloc((void **)&rp64, (size_t)(V + 1) * 8, dev)) != AG_OK) { ag_graph_free(g0); return s; }
+    cudaMemcpy(rp64, row_ptr, (size_t)(V + 1) * 8, cudaMemcpyDefault);
+    const uint32_t *gw = nullptr;
+    uint32_t *wtmp = nullptr;
+    if (weights) {  // the store keeps only interleaved (col,w); take the weights from the caller again
+        if ((s = dev_alloc((void **)&wtmp, E * 4 + 128, dev)) != AG_OK) { ag_graph_free(g0); dev_free(rp64, (size_t)(V + 1) * 8, dev); return s; }
+        cudaMemcpy(wtmp, weights, E * 4, cudaMemcpyDefault);
+        gw = wtmp;
+    }
+    void *tmp = nullptr;
+    size_t tb = 0;
+    auto cleanup = [&]() {
+        dev_free(rp64, (size_t)(V + 1) * 8, dev);
+        dev_free(cnt, (size_t)(V + 1) * 8, dev);
+        dev_free(wtmp, E * 4 + 128, dev);
+        dev_free(tmp, tb, dev);
+        ag_graph_free(g0);
+    };
+    if ((s = dev_alloc((void **)&cnt, (size_t)(V + 1) * 8, dev)) != AG_OK) { cleanup(); return s; }
+    if ((s = dev_alloc((void **)&nrp, (size_t)(V + 1) * 8, dev)) != AG_OK) { cleanup(); return s; }
+    dist_count_kernel<<<grid, 256>>>(rp64, g0->d_col, V, b, e, cnt);
+    cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, nrp, (int)V + 1);
+    if ((s = dev_alloc(&tmp, tb, dev)) != AG_OK) { dev_free(nrp, (size_t)(V + 1) * 8, dev); cleanup(); return s; }
+    cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, nrp, (int)V + 1);
+    uint64_t El = 0;
+    cudaMemcpy(&El, nrp + V, 8, cudaMemcpyDeviceToHost);
+    if ((s = dev_alloc((void **)&ncol, El * 4 + 128, dev)) != AG_OK) { dev_free(nrp, (size_t)(V + 1) * 8, dev); cleanup(); return s; }
+    if (gw && (s = dev_alloc((void **)&nw, El * 4 + 128, dev)) != AG_OK) {
+        dev_free(ncol, El * 4 + 128, dev);
+        dev_free(nrp, (size_t)(V + 1) * 8, dev);
+        cleanup();
+        return s;
+    }
+    dist_scatter_kernel<<<grid, 256>>>(rp64, g0->d_col, gw, V, b, e, nrp, ncol, nw);
+    note_launch(3);
+    cudaError_t ce = cudaDeviceSynchronize();
+    cleanup();
+    if (ce != cudaSuccess) {
+        dev_free(ncol, El * 4 + 128, dev);
+        dev_free(nw, El * 4 + 128, dev);
+        dev_free(nrp, (size_t)(V + 1) * 8, dev);
+        return cuda_status(ce, "dist partition");
+    }
+    // the local part is an ordinary graph handle (rows over all V, owned destinations only)
+    ag_graph gl = nullptr;
+    s = ag_graph_load_csr_ex(V, El, nrp, ncol, nw, dev, AG_LAYOUT_IDENTITY, &gl);
+    dev_free(ncol, El * 4 + 128, dev);
+    dev_free(nw, El * 4 + 128, dev);
+    dev_free(nrp, (size_t)(V + 1) * 8, dev);
+    if (s != AG_OK) return s;
+    if ((s = part_alloc(gl, c)) != AG_OK) { ag_graph_free(gl); return s; }
+    if (c->group) c->group->parts[c->rank] = gl;
+    *out_local = gl;
+    return AG_OK;
+}
+
+ag_status ag_dist_graph_load_local(ag_comm c, uint32_t V, uint64_t E_local, const uint64_t *row_ptr,
+                                   const uint32_t *col_idx, const uint32_t *weights, ag_graph *out_local) {
+    if (!c || !out_local) return set_error(AG_ERR_INVALID_ARG, "NULL argument");
+    *out_local = nullptr;
+    ag_graph gl = nullptr;
+    ag_status s = ag_graph_load_csr_ex(V, E_local, row_ptr, col_idx, weights, c->device, AG_LAYOUT_IDENTITY, &gl);
+    if (s != AG_OK) return s;
+    uint32_t b, e;
+    ag_dist_owned_range(V, c->rank, c->world, &b, &e);
+    unsigned *bad = nullptr;
+    if ((s = dev_alloc((void **)&bad, 16, c->device)) != AG_OK) { ag_graph_free(gl); return s; }
+    cudaMemset(bad, 0, 4);
+    if (E_local) owned_check_kernel<<<gl->num_sms * 4, 256>>>(gl->d_col, E_local, b, e, bad);
+    note_launch(1);
+    unsigned h = 0;
+    cudaMemcpy(&h, bad, 4, cudaMemcpyDeviceToHost);
+    dev_free(bad, 16, c->device);
+    if (h) { ag_graph_free(gl); return set_error(AG_ERR_BAD_CSR, "local CSR has a destination outside [%u, %u)", b, e); }
+    if ((s = part_alloc(gl, c)) != AG_OK) { ag_graph_free(gl); return s; }
+    if (c->group) c->group->parts[c->rank] = gl;
+    *out_local = gl;
+    return AG_OK;
+}
+
+}  // extern "C"
+
+namespace {
+
+// Lock-step driver over the participating ranks of THIS process (1 rank for NCCL, all for a group).
+ag_status dist_bfs_driver(std::vector<ag_graph_s *> &parts, uint32_t src, uint32_t **levels_owned,
+                          uint32_t **parents_owned, ag_run_stats *stats, cudaStream_t st) {
+    const int P = (int)parts.size();
+    ag_status s;
+    for (auto *g : parts) {
+        cudaSetDevice(g->device);
+        if ((s = dist_scratch(g)) != AG_OK) return s;
+        if (parents_owned && !g->d_lpar && (s = dev_alloc((void **)&g->d_lpar, (size_t)g->V * 4 + 128, g->device)) != AG_OK)
+            return s;
+    }
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    if (stats) {
+        cudaEventCreate(&e0);
+        cudaEventCreate(&e1);
+        cudaEventRecord(e0, st);
+    }
+    const uint32_t V = parts[0]->V;
+    for (auto *g : parts) {
+        ag_dist_part *d = g->dist;
+        dist_init_kernel<<<g->num_sms * 4, 256, 0, st>>>(g->d_level, parents_owned ? g->d_lpar : nullptr, g->d_vis,
+                                                        d->d_front, d->d_next, V, d->gwords, src);
+        cudaMemsetAsync(g->d_ctl, 0, offsetof(Ctl, q_len), st);   // no-op for the barrier word (self-resetting)
+        cudaMemsetAsync((char *)g->d_ctl + offsetof(Ctl, vexp), 0, 16, st);
+        note_launch(1);
+    }
+    uint32_t L = 0;
+    uint64_t front_n = 1;
+    uint32_t tcap = stats ? stats->trace_cap : 0;
+    for (;; ++L) {
+        if (stats && L < tcap && stats->trace_ws) stats->trace_ws[L] = (uint32_t)front_n;
+        for (auto *g : parts)
+            if ((s = run_level(g, L, parents_owned ? g->d_lpar : nullptr, st)) != AG_OK) return s;
+        // exchange: every rank contributes its owned slice of the next bitmap
+        if (P == 1 && parts[0]->dist->comm->nccl) {
+            ag_graph_s *g = parts[0];
+            ag_dist_part *d = g->dist;
+            ncclResult_t r = g_nccl.AllGather(d->d_next + (size_t)d->comm->rank * (d->S / 32), d->d_front, d->S / 8,
+                                              ncclUint8, d->comm->nccl, st);
+            if ((s = nccl_status(r, "ncclAllGather")) != AG_OK) return s;
+        } else {
+            for (auto *gd : parts) {
+                for (auto *gs : parts) {
+                    ag_dist_part *dd = gd->dist, *ds = gs->dist;
+                    const size_t off = (size_t)ds->comm->rank * (ds->S / 32);
+                    cudaMemcpyAsync(dd->d_front + off, ds->d_next + off, ds->S / 8, cudaMemcpyDeviceToDevice, st);
+                }
+            }
+        }
+        // clear the owned next slices, count the gathered frontier (every rank sees the same count)
+        ag_graph_s *g0 = parts[0];
+        for (auto *g : parts) {
+            ag_dist_part *d = g->dist;
+            cudaMemsetAsync(d->d_next + (size_t)d->comm->rank * (d->S / 32), 0, d->S / 8, st);
+        }
+        cudaMemsetAsync(g0->dist->d_cnt, 0, 8, st);
+        popcount_kernel<<<g0->num_sms * 2, 256, 0, st>>>(g0->dist->d_front, g0->dist->gwords, g0->dist->d_cnt);
+        note_launch(1);
+        cudaMemcpyAsync(g0->dist->h_cnt, g0->dist->d_cnt, 8, cudaMemcpyDeviceToHost, st);
+        cudaError_t ce = cudaStreamSynchronize(st);
+        if (ce != cudaSuccess) return cuda_status(ce, "dist level");
+        front_n = *g0->dist->h_cnt;
+        if (front_n == 0 || L > V) break;
+    }
+    // outputs: owned slices of level / parent
+    for (int r = 0; r < P; ++r) {
+        ag_graph_s *g = parts[r];
+        ag_dist_part *d = g->dist;
+        const size_t n = d->own_e - d->own_b;
+        if (levels_owned && levels_owned[r] && n)
+            cudaMemcpyAsync(levels_owned[r], g->d_level + d->own_b, n * 4, cudaMemcpyDefault, st);
+        if (parents_owned && parents_owned[r] && n)
+            cudaMemcpyAsync(parents_owned[r], g->d_lpar + d->own_b, n * 4, cudaMemcpyDefault, st);
+    }
+    if (stats) cudaEventRecord(e1, st);
+    cudaError_t ce = cudaStreamSynchronize(st);
+    if (ce != cudaSuccess) return cuda_status(ce, "dist bfs");
+    if (stats) {
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        cudaEventDestroy(e0);
+        cudaEventDestroy(e1);
+        stats->iterations = L + 1;
+        stats->device_ms = ms;
+        unsigned long long vx = 0, ex = 0;
+        for (auto *g : parts) {
+            Ctl c;
+            cudaMemcpy(&c, g->d_ctl, sizeof c, cudaMemcpyDeviceToHost);
+            vx += c.vexp;
+            ex += c.eexp;
+        }
+        stats->vertices_expanded = vx;  // summed over the ranks of this process
+        stats->edges_inspected = ex;
+        stats->trace_len = (L + 1) < tcap ? (L + 1) : tcap;
+    }
+    return AG_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+ag_status ag_dist_bfs(ag_graph local, uint32_t src, uint32_t *levels_owned, uint32_t *parents_owned,
+                      const ag_policy *policy, ag_run_stats *stats, void *stream) {
+    (void)policy;
+    if (!local || !local->dist) return set_error(AG_ERR_INVALID_ARG, "not a distributed graph");
+    if (src >= local->V) return set_error(AG_ERR_SRC_RANGE, "src %u >= V %u", src, local->V);
+    if (stats && stats->struct_size != sizeof(ag_run_stats)) return set_error(AG_ERR_INVALID_ARG, "stats size");
+    if (local->dist->comm->group) return set_error(AG_ERR_INVALID_ARG, "virtual-group graph: use ag_dist_bfs_group");
+    std::vector<ag_graph_s *> parts{local};
+    uint32_t *lv[1] = {levels_owned};
+    uint32_t *pa[1] = {parents_owned};
+    cudaSetDevice(local->device);
+    return dist_bfs_driver(parts, src, lv, parents_owned ? pa : nullptr, stats, (cudaStream_t)stream);
+}
+
+ag_status ag_dist_bfs_group(ag_graph *locals, int world, uint32_t src, uint32_t **levels_owned,
+                            uint32_t **parents_owned, ag_run_stats *stats, void *stream) {
+    if (!locals || world < 1) return set_error(AG_ERR_INVALID_ARG, "bad args");
+    std::vector<ag_graph_s *> parts;
+    for (int r = 0; r < world; ++r) {
+        if (!locals[r] || !locals[r]->dist || !locals[r]->dist->comm->group || locals[r]->dist->comm->rank != r)
+            return set_error(AG_ERR_INVALID_ARG, "locals[%d] is not rank %d of a virtual group", r, r);
+        parts.push_back(locals[r]);
+    }
+    if (src >= parts[0]->V) return set_error(AG_ERR_SRC_RANGE, "src out of range");
+    if (stats && stats->struct_size != sizeof(ag_run_stats)) return set_error(AG_ERR_INVALID_ARG, "stats size");
+    cudaSetDevice(parts[0]->device);
+    return dist_bfs_driver(parts, src, levels_owned, parents_owned, stats, (cudaStream_t)stream);
 }
 
 }  // extern "C"
