@@ -264,9 +264,13 @@ ag_status check_policy(const ag_policy *p) {
 // ------------------------------------------------------------------------------------------------
 template <int ALG, int ORD, typename Off>
 static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t st) {
-    auto fn = traverse_kernel<ALG, ORD, Off>;
+    // the tuned adaptive policy runs the specialisation without the paper's static variants
+    const bool tuned = a.pol.kind == AG_POLICY_TUNED && a.pol.force_map == 0 && a.pol.force_ws == 0;
+    auto fn = tuned ? traverse_kernel<ALG, ORD, Off, true> : traverse_kernel<ALG, ORD, Off, false>;
+    const size_t dyn = 0;
+    if (dyn) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
     int occ = 0;
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, BS, 0);
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, BS, dyn);
     if (e != cudaSuccess || occ < 1) return cuda_status(e == cudaSuccess ? cudaErrorLaunchOutOfResources : e, "occupancy");
     a.nblocks = (uint32_t)(occ * g->num_sms);
     // Cooperative launch (co-resident grid for the software grid barrier) with an L2 access-policy
@@ -275,7 +279,7 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(a.nblocks);
     cfg.blockDim = dim3(BS);
-    cfg.dynamicSmemBytes = 0;
+    cfg.dynamicSmemBytes = dyn;
     cfg.stream = st;
     cudaLaunchAttribute attrs[2];
     attrs[0].id = cudaLaunchAttributeCooperative;

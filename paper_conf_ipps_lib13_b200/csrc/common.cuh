@@ -25,10 +25,16 @@ static_assert(LOG_BS > 0, "BS must be 128, 256, 512 or 1024");
 // Occupancy / batch depth per algorithm (measured on B200): BFS is best at 4 CTAs/SM
 // (64 regs) with 4-edge batches, SSSP (8-byte states, more atomics) at 8 CTAs/SM with 2-edge batches.
 #ifndef AG_MINB_BFS
-#define AG_MINB_BFS 4
+#define AG_MINB_BFS 5
 #endif
 #ifndef AG_MINB_SSSP
 #define AG_MINB_SSSP 8
+#endif
+#ifndef AG_MINB_BFS_T
+#define AG_MINB_BFS_T AG_MINB_BFS
+#endif
+#ifndef AG_MINB_SSSP_T
+#define AG_MINB_SSSP_T AG_MINB_SSSP
 #endif
 #ifndef AG_EB_BFS
 #define AG_EB_BFS 4
@@ -49,6 +55,12 @@ enum { WS_BM = 1, WS_QU = 2 };
 // HUB_CHUNK-edge tasks drained by all CTAs.
 #ifndef AG_HUBCHUNK
 #define AG_HUBCHUNK 4096
+#endif
+#ifndef AG_QB
+#define AG_QB 2           // hybrid mapping: aligned 16-byte pieces per thread per step (BFS)
+#endif
+#ifndef AG_QB_SSSP
+#define AG_QB_SSSP 1      //                                                  (SSSP)
 #endif
 #ifndef AG_LONG_MIN
 #define AG_LONG_MIN 512   // hybrid mapping: lists this long go to aligned warp windows
@@ -199,6 +211,45 @@ __device__ __forceinline__ void red_or(uint32_t *p, uint32_t v) {
 }
 
 __device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31u; }
+
+// ---- mbarrier + bulk async copy (TMA engine, cp.async.bulk -> SASS UBLKCP) ----
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t *mbar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(mbar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *mbar, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(mbar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t *mbar, unsigned parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok) : "r"(smem_u32(mbar)), "r"(parity) : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *mbar, unsigned parity) {
+    while (!mbar_try_wait(mbar, parity)) {
+    }
+}
+// cp.async (LDGSTS) 16-byte global -> shared, L1 bypass, with an L2 policy
+__device__ __forceinline__ void cp_async16(void *dst, const void *src, uint64_t) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+// bulk copy global -> shared (16-B aligned, size multiple of 16), completing tx bytes on mbar
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned bytes, uint64_t *mbar, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+        ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(mbar)), "l"(pol) : "memory");
+}
 __device__ __forceinline__ unsigned long long globaltimer_ns() {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));

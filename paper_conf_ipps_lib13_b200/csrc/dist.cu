@@ -213,7 +213,7 @@ __global__ void __launch_bounds__(BS, AG_MINB_BFS) dist_level_kernel(const TravA
         const uint32_t i = t * tile_n + threadIdx.x;
         const bool valid = threadIdx.x < tile_n && i < qn;
         const uint32_t u = valid ? a.q[0][i] : 0u;
-        if (__syncthreads_or(valid)) process_tile(ops, sm, MAP_H, valid, u, 32u, a.has_hubs != 0, slot, tag);
+        if (__syncthreads_or(valid)) process_tile<true>(ops, sm, MAP_H, valid, u, 32u, a.has_hubs != 0, slot, tag);
         t = sm.tnext[par];
         par ^= 1;
     }

@@ -66,7 +66,9 @@ struct TravArgs {
     uint32_t has_hubs;
 };
 
-constexpr int WQ_CAP = 32 * EB_MAX + 32;
+// per-warp staging capacity: one batch appends at most 32 x (edges per thread per batch), plus < 32 left over
+constexpr int BATCH_MAX = (EB_MAX > 4 * AG_QB) ? EB_MAX : 4 * AG_QB;
+constexpr int WQ_CAP = 32 * BATCH_MAX + 32;
 
 template <typename Off>
 struct __align__(16) TileSmem {
@@ -83,8 +85,7 @@ struct __align__(16) TileSmem {
     int redi[WARPS_PER_CTA];
     uint32_t tnext[2];
     uint32_t bcast;
-    uint32_t task;
-    uint32_t status;
+    uint32_t htask[2][4];   // hub-drain task slots (u, uval, chunk, status)
 };
 
 // ------------------------------------------------------------------------------------------------
@@ -252,6 +253,14 @@ struct Ops {
             return;
         }
 #endif
+        batch_vals<NB, STAGED>(u, uv, v, wt, ok);
+    }
+
+    // The status + update half of a batch, for neighbour ids already in registers.
+    template <int NB, bool STAGED>
+    __device__ __forceinline__ void batch_vals(const uint32_t (&u)[NB], const uint32_t (&uv)[NB], const uint32_t (&v)[NB],
+                                               const uint32_t (&wt)[NB], const bool (&ok)[NB]) {
+        St st[NB];
 #pragma unroll
         for (int j = 0; j < NB; ++j) st[j] = ok[j] ? status(v[j]) : (St)0;
 #if defined(AG_EXPERIMENT) && AG_EXPERIMENT == 2   // ceiling experiment: stream + status, no update
@@ -263,21 +272,73 @@ struct Ops {
             return;
         }
 #endif
+        if constexpr (STAGED) {
+            uint32_t nwm = 0;   // bit j: v[j] entered the next working set
 #pragma unroll
-        for (int j = 0; j < NB; ++j) {
-            bool nw = update(u[j], uv[j], v[j], wt[j], st[j], ok[j]);
-            if constexpr (STAGED) {
-                const unsigned m = __ballot_sync(0xffffffffu, nw);
-                if (nw) wbuf[wfill + __popc(m & ((1u << lane_id()) - 1u))] = v[j];
-                wfill += __popc(m);
-            } else {
+            for (int j = 0; j < NB; ++j) nwm |= update(u[j], uv[j], v[j], wt[j], st[j], ok[j]) ? (1u << j) : 0u;
+            if (__any_sync(0xffffffffu, nwm != 0)) {   // rare on the big levels: skip the ballots otherwise
+#pragma unroll
+                for (int j = 0; j < NB; ++j) {
+                    const bool nw = (nwm >> j) & 1u;
+                    const unsigned m = __ballot_sync(0xffffffffu, nw);
+                    if (nw) wbuf[wfill + __popc(m & ((1u << lane_id()) - 1u))] = v[j];
+                    wfill += __popc(m);
+                }
+                __syncwarp();
+                if (wfill >= 32) warp_flush(false);
+            }
+        } else {
+#pragma unroll
+            for (int j = 0; j < NB; ++j) {
+                bool nw = update(u[j], uv[j], v[j], wt[j], st[j], ok[j]);
                 warp_append(q_next, qlen_next, nw, v[j]);
             }
         }
-        if constexpr (STAGED) {
-            __syncwarp();
-            if (wfill >= 32) warp_flush(false);
+    }
+
+    // QB aligned 16-byte pieces per thread: piece q holds CSR entries [q*QE, q*QE + QE) (one 128-bit
+    // load), of which those in [lo, hi) (one adjacency list) are expanded.  All loads of the QB pieces
+    // are issued first, then all status loads, then the updates (warp-converged; staged appends).
+    static constexpr uint32_t QE = (ALG == ALG_SSSP) ? 2u : 4u;
+    static constexpr int QB = (ALG == ALG_SSSP) ? AG_QB_SSSP : AG_QB;
+    template <int NQ>
+    __device__ __forceinline__ void pieces(const uint32_t (&pu)[NQ], const uint32_t (&pv)[NQ], const Off (&pq)[NQ],
+                                           const Off (&plo)[NQ], const Off (&phi)[NQ], const bool (&pok)[NQ]) {
+        constexpr int N = NQ * (int)QE;
+        uint32_t uu[N], vv[N], v[N], wt[N];
+        bool ok[N];
+#pragma unroll
+        for (int j = 0; j < NQ; ++j) {
+            uint4 c = pok[j] ? ld_stream4(reinterpret_cast<const uint4 *>(
+                                              (ALG == ALG_SSSP) ? (const void *)(a.cw + pq[j] * QE)
+                                                                : (const void *)(a.col + pq[j] * QE)),
+                                          pol_stream)
+                             : make_uint4(0u, 0u, 0u, 0u);
+            const Off e0 = pq[j] * QE;
+            if constexpr (ALG == ALG_SSSP) {
+                v[2 * j] = c.x; wt[2 * j] = c.y; v[2 * j + 1] = c.z; wt[2 * j + 1] = c.w;
+            } else {
+                v[4 * j] = c.x; v[4 * j + 1] = c.y; v[4 * j + 2] = c.z; v[4 * j + 3] = c.w;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) wt[4 * j + k] = 1u;
+            }
+#pragma unroll
+            for (int k = 0; k < (int)QE; ++k) {
+                ok[j * QE + k] = pok[j] && e0 + k >= plo[j] && e0 + k < phi[j];
+                uu[j * QE + k] = pu[j];
+                vv[j * QE + k] = pv[j];
+            }
         }
+#if defined(AG_EXPERIMENT) && AG_EXPERIMENT == 1   // ceiling experiment: stream only
+        {
+            uint32_t acc = 0;
+#pragma unroll
+            for (int j = 0; j < N; ++j) acc += ok[j] ? v[j] : 0u;
+            if (acc == 0xFFFFFFFFu) ovf = true;
+            return;
+        }
+#endif
+        batch_vals<N, true>(uu, vv, v, wt, ok);
     }
 
     // One aligned window of WIN = 32 x EPL consecutive CSR entries [wbase, wbase + WIN), restricted to
@@ -410,11 +471,10 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, Tile
 // ------------------------------------------------------------------------------------------------
 // One tile: thread tid holds working-set element (valid, u).  Applies the mapping.
 // ------------------------------------------------------------------------------------------------
-template <int ALG, int ORD, typename Off>
+template <bool TUNED, int ALG, int ORD, typename Off>
 __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<Off> &sm, uint32_t map,
                                              bool valid, uint32_t u, uint32_t group, bool hubs, uint32_t slot,
                                              uint32_t tag) {
-    constexpr int EB = Ops<ALG, ORD, Off>::EB;
     const TravArgs<Off> &a = ops.a;
     Off beg = 0;
     uint32_t deg = 0, uval = 0;
@@ -426,7 +486,7 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<O
         if (ex) ops.edges_thread(u, uval, beg, deg);
         return;
     }
-    if (map == MAP_W || (map == MAP_B && group == 32)) {
+    if (!TUNED && (map == MAP_W || (map == MAP_B && group == 32))) {
         unsigned m = __ballot_sync(0xffffffffu, ex && deg > 0);
         while (m) {
             const int j = __ffs(m) - 1;
@@ -439,7 +499,7 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<O
         }
         return;
     }
-    if (map == MAP_B) {
+    if (!TUNED && map == MAP_B) {
         sm.u[tid] = u;
         sm.uval[tid] = uval;
         sm.deg[tid] = deg;
@@ -477,77 +537,57 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<O
             }
         }
     }
-    // short lists (< 32 entries) -> packed gather; long lists -> aligned warp windows
-    constexpr uint32_t WIN = Ops<ALG, ORD, Off>::WIN;
-    const bool is_long = !is_hub && deg >= (uint32_t)AG_LONG_MIN;
-    const uint32_t d = (!is_hub && !is_long) ? deg : 0u;
-    const uint32_t nw = is_long ? (uint32_t)((beg + deg + WIN - 1) / WIN - beg / WIN) : 0u;
-    // CTA-wide exclusive scans of (short degrees, long-list window counts), packed in one u32 pair
-    uint32_t x = d, y = nw;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        uint32_t xo = __shfl_up_sync(0xffffffffu, x, o), yo = __shfl_up_sync(0xffffffffu, y, o);
-        if (lane >= (unsigned)o) { x += xo; y += yo; }
-    }
-    if (lane == 31) { sm.red32[0][tid >> 5] = x; sm.red32[1][tid >> 5] = y; }
-    __syncthreads();
-    if (tid < 32) {
-        uint32_t wv = (tid < (unsigned)WARPS_PER_CTA) ? sm.red32[0][tid] : 0, wx = wv;
-        uint32_t zv = (tid < (unsigned)WARPS_PER_CTA) ? sm.red32[1][tid] : 0, zx = zv;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            uint32_t t1 = __shfl_up_sync(0xffffffffu, wx, o), t2 = __shfl_up_sync(0xffffffffu, zx, o);
-            if (tid >= (unsigned)o) { wx += t1; zx += t2; }
-        }
-        if (tid < (unsigned)WARPS_PER_CTA) { sm.woff[0][tid] = wx - wv; sm.woff[1][tid] = zx - zv; }
-    }
-    __syncthreads();
-    const uint32_t excl = sm.woff[0][tid >> 5] + x - d;
-    const uint32_t wexcl = sm.woff[1][tid >> 5] + y - nw;
-    sm.scan[tid] = excl;
-    sm.wscan[tid] = wexcl;
+    // every (non-hub) adjacency list is cut into aligned 16-byte pieces (QE entries each: 4 col ids for
+    // BFS, 2 (col, w) pairs for SSSP); a CTA scan of the piece counts gives each thread QB pieces per
+    // step: one owner search + one 128-bit load per piece, coalesced across the warp
+    constexpr uint32_t QE = Ops<ALG, ORD, Off>::QE;
+    const uint32_t d = is_hub ? 0u : deg;
+    const uint32_t np = d ? (uint32_t)((beg + d + QE - 1) / QE - beg / QE) : 0u;
+    // (the __syncthreads_or that opened this tile guarantees nobody still reads the previous tile)
     sm.u[tid] = u;
     sm.uval[tid] = uval;
     sm.beg[tid] = beg;
-    sm.deg[tid] = deg;
-    if (tid == BS - 1) { sm.scan[BS] = excl + d; sm.wscan[BS] = wexcl + nw; }
-    __syncthreads();
-    // long lists: warps take windows round-robin (owner by binary search, once per window)
-    const uint32_t NWIN = sm.wscan[BS];
-    for (uint32_t wi = tid >> 5; wi < NWIN; wi += WARPS_PER_CTA) {
-        uint32_t lo = 0, hi = BS;
+    sm.deg[tid] = d;
+    uint32_t x = np;
 #pragma unroll
-        for (int step = 0; step < LOG_BS; ++step) {
-            uint32_t mid = (lo + hi) >> 1;
-            if (sm.wscan[mid] <= wi) lo = mid; else hi = mid;
-        }
-        const Off b0 = sm.beg[lo];
-        const Off wbase = (b0 / WIN + (wi - sm.wscan[lo])) * WIN;
-        ops.window(sm.u[lo], sm.uval[lo], wbase, b0, b0 + sm.deg[lo]);
+    for (int o = 1; o < 32; o <<= 1) {
+        uint32_t xo = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= (unsigned)o) x += xo;
     }
-    // short lists: packed, load-balanced gather
-    const uint32_t S = sm.scan[BS];
-    for (uint32_t base = 0; base < S; base += EB * BS) {
-        uint32_t uu[EB], vv[EB];
-        Off e[EB];
-        bool ok[EB];
+    if (lane == 31) sm.red32[0][tid >> 5] = x;
+    __syncthreads();
+    uint32_t woff = 0;   // every thread sums the preceding warps' totals (broadcast reads)
+    for (uint32_t w = 0; w < (tid >> 5); ++w) woff += sm.red32[0][w];
+    const uint32_t excl = woff + x - np;
+    sm.scan[tid] = excl;
+    if (tid == BS - 1) sm.scan[BS] = excl + np;
+    __syncthreads();
+    const uint32_t NP = sm.scan[BS];
+    constexpr int QB = Ops<ALG, ORD, Off>::QB;
+    for (uint32_t base = 0; base < NP; base += QB * BS) {
+        uint32_t pu[QB], pv[QB];
+        Off pq[QB], plo[QB], phi[QB];
+        bool pok[QB];
 #pragma unroll
-        for (int j = 0; j < EB; ++j) {
-            const uint32_t k = base + j * BS + tid;
-            ok[j] = k < S;
-            uint32_t lo = 0, hi = BS;  // owner: the largest i with scan[i] <= k
+        for (int j = 0; j < QB; ++j) {
+            const uint32_t p = base + j * BS + tid;
+            pok[j] = p < NP;
+            uint32_t lo = 0, hi = BS;   // owner: the largest i with scan[i] <= p
 #pragma unroll
             for (int step = 0; step < LOG_BS; ++step) {
-                uint32_t mid = (lo + hi) >> 1;
-                if (sm.scan[mid] <= k) lo = mid; else hi = mid;
+                const uint32_t mid = (lo + hi) >> 1;
+                if (sm.scan[mid] <= p) lo = mid; else hi = mid;
             }
-            uu[j] = sm.u[lo];
-            vv[j] = sm.uval[lo];
-            e[j] = sm.beg[lo] + (k - sm.scan[lo]);
+            pu[j] = sm.u[lo];
+            pv[j] = sm.uval[lo];
+            const Off bo = sm.beg[lo];
+            plo[j] = bo;
+            phi[j] = bo + sm.deg[lo];
+            pq[j] = bo / QE + (p - sm.scan[lo]);   // aligned piece index
         }
-        ops.template batch<EB, true>(uu, vv, e, ok);
+        ops.template pieces<QB>(pu, pv, pq, plo, phi, pok);
     }
-    __syncthreads();
+    // no trailing barrier: the next tile's __syncthreads_or orders the reuse of the tile arrays
 }
 
 // drain the hub-chunk tasks of this iteration (hybrid mapping)
@@ -561,9 +601,14 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, TileSmem<Off
         __threadfence();
         atomicAdd(&ctl->stage_done[slot], 1u);
     }
+    // the leader claims task indices one ahead (the claim's round trip overlaps the previous task);
+    // tasks are handed to the CTA through two shared-memory slots, one barrier per task
+    uint32_t claimed = 0;
+    if (threadIdx.x == 0) claimed = atomicAdd(&ctl->hub_head[slot], 1u);
+    int par = 0;
     for (;;) {
         if (threadIdx.x == 0) {
-            uint32_t t = atomicAdd(&ctl->hub_head[slot], 1u);
+            const uint32_t t = claimed;
             uint32_t status = 0;  // 0 = done, 1 = ready
             for (;;) {
                 uint32_t tail = ld_acquire(&ctl->hub_tail[slot]);
@@ -580,21 +625,40 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, TileSmem<Off
                 }
                 __nanosleep(64);
             }
-            sm.task = t;
-            sm.status = status;
+            if (status) {
+                const uint32_t *tk = a.hub + 4ull * t;
+                sm.htask[par][0] = tk[0];
+                sm.htask[par][1] = tk[1];
+                sm.htask[par][2] = tk[2];
+                claimed = atomicAdd(&ctl->hub_head[slot], 1u);   // prefetch the next claim
+            }
+            sm.htask[par][3] = status;
         }
         __syncthreads();
-        const uint32_t t = sm.task, st = sm.status;
-        __syncthreads();
-        if (!st) break;
-        const uint32_t *tk = a.hub + 4ull * t;
-        const uint32_t u = tk[0], uval = tk[1], k = tk[2];
+        if (!sm.htask[par][3]) break;
+        const uint32_t u = sm.htask[par][0], uval = sm.htask[par][1], k = sm.htask[par][2];
+        par ^= 1;
         const Off b0 = a.rp[u], e0 = a.rp[u + 1];
         const Off b = b0 + (Off)k * HUB_CHUNK;
         const Off e = (e0 - b > (Off)HUB_CHUNK) ? b + HUB_CHUNK : e0;
-        constexpr uint32_t WIN = Ops<ALG, ORD, Off>::WIN;
-        const Off w0 = b / WIN, w1 = (e + WIN - 1) / WIN;
-        for (Off wi = w0 + (threadIdx.x >> 5); wi < w1; wi += WARPS_PER_CTA) ops.window(u, uval, wi * WIN, b, e);
+        constexpr uint32_t QE = Ops<ALG, ORD, Off>::QE;
+        constexpr int QB = Ops<ALG, ORD, Off>::QB;
+        const Off q0 = b / QE, q1 = (e + QE - 1) / QE;
+        for (Off qb = q0; qb < q1; qb += (Off)QB * BS) {
+            uint32_t pu[QB], pv[QB];
+            Off pq[QB], plo[QB], phi[QB];
+            bool pok[QB];
+#pragma unroll
+            for (int j = 0; j < QB; ++j) {
+                pq[j] = qb + (Off)(j * BS + threadIdx.x);
+                pok[j] = pq[j] < q1;
+                pu[j] = u;
+                pv[j] = uval;
+                plo[j] = b;
+                phi[j] = e;
+            }
+            ops.template pieces<QB>(pu, pv, pq, plo, phi, pok);
+        }
     }
 }
 
@@ -629,10 +693,14 @@ __device__ __forceinline__ void compact_bitmap(const uint32_t *bm, uint32_t nwor
 // ------------------------------------------------------------------------------------------------
 // The persistent kernel
 // ------------------------------------------------------------------------------------------------
-template <int ALG, int ORD, typename Off>
-__global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? AG_MINB_SSSP : AG_MINB_BFS)
+// TUNED = the adaptive B200 policy only (thread / hybrid mappings over the queue): the paper's
+// static variants are compiled out, which frees registers for occupancy.
+template <int ALG, int ORD, typename Off, bool TUNED>
+__global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T : AG_MINB_SSSP)
+                                                      : (TUNED ? AG_MINB_BFS_T : AG_MINB_BFS))
     traverse_kernel(const TravArgs<Off> a) {
     __shared__ TileSmem<Off> sm;
+
     Ctl *ctl = a.ctl;
     const uint32_t gtid = blockIdx.x * BS + threadIdx.x, gthreads = a.nblocks * BS;
     const uint32_t src = a.inv ? a.inv[a.src] : a.src;
@@ -697,7 +765,8 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? AG_MINB_SSSP : AG_MINB_B
         if (n == 0 || it >= a.max_iters) break;
         // decision maker, re-evaluated every sample_every iterations (inspector sampling, 26.s7-9)
         const uint8_t var = (it % a.pol.sample_every == 0 || prev_var == 0) ? select_variant(a.pol, n, 0) : prev_var;
-        const uint32_t map = var >> 2, ws = var & 3;
+        const uint32_t map = TUNED ? ((var >> 2) == MAP_T ? (uint32_t)MAP_T : (uint32_t)MAP_H) : (var >> 2);
+        const uint32_t ws = TUNED ? (uint32_t)WS_QU : (var & 3u);
         const uint32_t tag = a.epoch * 0x9E3779B1u + it + 1;
         if (blockIdx.x == 0 && threadIdx.x == 0) {
             if (it < a.trace_cap && a.trace_ws) {
@@ -763,26 +832,28 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? AG_MINB_SSSP : AG_MINB_B
         const uint32_t ntiles = (ws == WS_BM) ? (a.V + BS - 1) / BS : (qn + tile_n - 1) / tile_n;
         const bool hubs = (map == MAP_H) && a.has_hubs;
 
-        // dynamic tile scheduler: first tile static, then one atomic per tile, fetched one tile ahead
-        // (double-buffered in smem; the __syncthreads_or below orders the write before the read)
-        uint32_t t = blockIdx.x;
-        int par = 0;
-        while (t < ntiles) {
-            if (threadIdx.x == 0) sm.tnext[par] = a.nblocks + atomicAdd(&ctl->tile_ctr[slot], 1u);
-            bool valid;
-            uint32_t u;
-            if (ws == WS_BM) {
-                u = t * BS + threadIdx.x;
-                valid = u < a.V && ((bmc[u >> 5] >> (u & 31)) & 1u);
-            } else {
-                uint32_t i = t * tile_n + s_idx;
-                valid = s_idx < tile_n && i < qn;
-                u = valid ? qc[i] : 0u;
+        {
+            // dynamic tile scheduler: first tile static, then one atomic per tile, fetched one tile ahead
+            // (double-buffered in smem; the __syncthreads_or below orders the write before the read)
+            uint32_t t = blockIdx.x;
+            int par = 0;
+            while (t < ntiles) {
+                if (threadIdx.x == 0) sm.tnext[par] = a.nblocks + atomicAdd(&ctl->tile_ctr[slot], 1u);
+                bool valid;
+                uint32_t u;
+                if (ws == WS_BM) {
+                    u = t * BS + threadIdx.x;
+                    valid = u < a.V && ((bmc[u >> 5] >> (u & 31)) & 1u);
+                } else {
+                    uint32_t i = t * tile_n + s_idx;
+                    valid = s_idx < tile_n && i < qn;
+                    u = valid ? qc[i] : 0u;
+                }
+                if (__syncthreads_or(valid))  // skip empty tiles (sparse bitmap): uniform branch
+                    process_tile<TUNED>(ops, sm, map, valid, u, a.pol.cta_group, hubs, slot, tag);
+                t = sm.tnext[par];
+                par ^= 1;
             }
-            if (__syncthreads_or(valid))  // skip empty tiles (sparse bitmap): uniform branch
-                process_tile(ops, sm, map, valid, u, a.pol.cta_group, hubs, slot, tag);
-            t = sm.tnext[par];
-            par ^= 1;
         }
         if (hubs) drain_hubs(ops, sm, slot, tag);
         ops.warp_flush(true);
