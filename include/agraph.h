@@ -34,6 +34,7 @@ extern "C" {
 
 #define AG_ABI_VERSION 1u
 #define AG_INF 0xFFFFFFFFu
+#define AG_WINDOW_AUTO 0xFFFFFFFFu
 
 typedef struct ag_graph_s *ag_graph; /* opaque, library-owned device CSR + scratch */
 typedef struct ag_comm_s *ag_comm;   /* opaque multi-GPU communicator (one per process/GPU) */
@@ -86,7 +87,10 @@ typedef struct {
     uint32_t delta;          /* ordered-SSSP bucket width; 1 = the paper's Dijkstra batches (28.s8, R9) */
     uint32_t thread_tpb;     /* thread-mapping block size used for T2, paper 192 (26.s27) */
     uint32_t cta_group;      /* block-mapping group size (multiple of 32); 0 = auto (26.s28, R16) */
-    uint32_t reserved[4];    /* must be 0 */
+    uint32_t sssp_window;    /* unordered SSSP: expand only frontier vertices with dist < min + window
+                                (others stay in the working set); 0 = off (plain Bellman-Ford rounds);
+                                AG_WINDOW_AUTO = tuned: off on skewed graphs, else 8 x max_weight / avg degree */
+    uint32_t reserved[3];    /* must be 0 */
 } ag_policy;
 
 typedef struct {
@@ -100,6 +104,8 @@ typedef struct {
     uint32_t num_sms;            /* SM count of that device */
     uint32_t offset_bytes;       /* 4 if row offsets are stored as u32 (E < 2^32), else 8 */
     uint32_t layout;             /* ag_layout actually used (IDENTITY or DEGREE) */
+    uint32_t max_weight;         /* largest edge weight (0 if unweighted) */
+    uint32_t reserved2;
 } ag_graph_info;
 
 /* Device vertex layout.  DEGREE relabels vertices by descending out-degree at load
@@ -133,7 +139,8 @@ typedef struct {
  * ------------------------------------------------------------------------------------------- */
 
 /* Fill *p with defaults for `device`: order UNORDERED, mapping/workset AUTO, kind TUNED,
- * T1 = 32, thread_tpb = 192, T2 = 192 x #SMs, t3_ppm = 15625, delta = 1, sample_every = 1.
+ * T1 = 32, thread_tpb = 192, T2 = 192 x #SMs, t3_ppm = 15625, delta = 1, sample_every = 1,
+ * sssp_window = AG_WINDOW_AUTO.
  * Errors: AG_ERR_INVALID_ARG (p NULL), AG_ERR_NO_DEVICE. */
 ag_status ag_policy_default(ag_policy *p, int device);
 

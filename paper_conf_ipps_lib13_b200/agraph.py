@@ -23,6 +23,7 @@ MAP_AUTO, MAP_THREAD, MAP_WARP, MAP_CTA, MAP_HYBRID = 0, 1, 2, 3, 4
 WS_AUTO, WS_BITMAP, WS_QUEUE = 0, 1, 2
 POLICY_PAPER, POLICY_TUNED = 0, 1
 LAYOUT_AUTO, LAYOUT_IDENTITY, LAYOUT_DEGREE = 0, 1, 2
+WINDOW_AUTO = 0xFFFFFFFF
 STATUS = {0: "AG_OK", 1: "AG_ERR_INVALID_ARG", 2: "AG_ERR_BAD_CSR", 3: "AG_ERR_SRC_RANGE", 4: "AG_ERR_NO_WEIGHTS",
           5: "AG_ERR_OVERFLOW", 6: "AG_ERR_OOM", 7: "AG_ERR_CUDA", 8: "AG_ERR_NCCL", 9: "AG_ERR_UNSUPPORTED",
           10: "AG_ERR_NO_DEVICE"}
@@ -50,14 +51,15 @@ class Policy(ctypes.Structure):
                 ("workset", ctypes.c_uint32), ("kind", ctypes.c_uint32), ("t1_avg_degree", ctypes.c_uint32),
                 ("t2_ws", ctypes.c_uint64), ("t3_ppm", ctypes.c_uint32), ("sample_every", ctypes.c_uint32),
                 ("delta", ctypes.c_uint32), ("thread_tpb", ctypes.c_uint32), ("cta_group", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32 * 4)]
+                ("sssp_window", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3)]
 
 
 class GraphInfo(ctypes.Structure):
     _fields_ = [("num_vertices", ctypes.c_uint32), ("min_deg", ctypes.c_uint32), ("max_deg", ctypes.c_uint32),
                 ("num_edges", ctypes.c_uint64), ("deg_sum", ctypes.c_uint64), ("isolated", ctypes.c_uint32),
                 ("weighted", ctypes.c_uint32), ("device", ctypes.c_int32), ("num_sms", ctypes.c_uint32),
-                ("offset_bytes", ctypes.c_uint32), ("layout", ctypes.c_uint32)]
+                ("offset_bytes", ctypes.c_uint32), ("layout", ctypes.c_uint32), ("max_weight", ctypes.c_uint32),
+                ("reserved2", ctypes.c_uint32)]
 
 
 class RunStats(ctypes.Structure):

@@ -101,6 +101,7 @@ ag_status check_device(int device, int *num_sms) {
 struct LoadStats {
     unsigned int bad;            // bit 0 rp[0], 1 monotone, 2 rp[V], 3 col range, 4 weight range
     unsigned int min_deg, max_deg, isolated;
+    unsigned int max_w;
 };
 
 __global__ void validate_rows_kernel(const uint64_t *rp, uint32_t V, uint64_t E, LoadStats *st) {
@@ -131,16 +132,21 @@ __global__ void validate_rows_kernel(const uint64_t *rp, uint32_t V, uint64_t E,
 }
 
 __global__ void validate_edges_kernel(const uint32_t *col, const uint32_t *w, uint64_t E, uint32_t V, LoadStats *st) {
-    unsigned bad = 0;
+    unsigned bad = 0, mw = 0;
     for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < E; e += (uint64_t)gridDim.x * blockDim.x) {
         if (col[e] >= V) bad |= 8;
         if (w) {
             uint32_t x = w[e];
             if (x == 0 || x >= 0x80000000u) bad |= 16;
+            mw = max(mw, x);
         }
     }
     bad = __reduce_or_sync(0xffffffffu, bad);
-    if ((threadIdx.x & 31) == 0 && bad) atomicOr(&st->bad, bad);
+    mw = __reduce_max_sync(0xffffffffu, mw);
+    if ((threadIdx.x & 31) == 0) {
+        if (bad) atomicOr(&st->bad, bad);
+        if (mw) atomicMax(&st->max_w, mw);
+    }
 }
 
 __global__ void interleave_kernel(const uint32_t *col, const uint32_t *w, uint2 *cw, uint64_t E) {
@@ -241,6 +247,18 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
     grp = grp > (uint32_t)BS ? (uint32_t)BS : grp;
     grp &= ~31u;
     d.cta_group = grp;
+    if (p.sssp_window == AG_WINDOW_AUTO) {
+        // tuned: Bellman-Ford re-expansion is distance-ordering waste on long-path graphs (grid: 152x,
+        // ER: 4.3x) but not on power-law graphs (R-MAT: no gain) -- measured with tools/sweep.py
+        const uint64_t avg = g.V ? (g.E + g.V - 1) / g.V : 1;
+        const bool skewed = g.info.layout == AG_LAYOUT_DEGREE;
+        uint64_t w = 8ull * g.info.max_weight / (avg ? avg : 1);
+        if (w < 1) w = 1;
+        if (w > 0x7FFFFFFFull) w = 0x7FFFFFFFull;
+        d.window = (p.kind == AG_POLICY_TUNED && !skewed && g.info.max_weight) ? (uint32_t)w : 0u;
+    } else {
+        d.window = p.sssp_window;
+    }
     d.V = g.V;
     d.E = g.E;
     d.max_deg = g.info.max_deg;
@@ -503,6 +521,7 @@ ag_status ag_policy_default(ag_policy *p, int device) {
     p->sample_every = 1;
     p->delta = 1;
     p->cta_group = 0;
+    p->sssp_window = AG_WINDOW_AUTO;
     return AG_OK;
 }
 
@@ -557,7 +576,7 @@ ag_status ag_graph_load_csr_ex(uint32_t V, uint64_t E, const uint64_t *row_ptr, 
     cudaError_t e = cudaMemcpy(rp64, row_ptr, (size_t)(V + 1) * 8, cudaMemcpyDefault);
     if (e == cudaSuccess && E) e = cudaMemcpy(g->d_col, col_idx, E * 4, cudaMemcpyDefault);
     if (e == cudaSuccess && E && weights) e = cudaMemcpy(g->d_w, weights, E * 4, cudaMemcpyDefault);
-    LoadStats hs = {0, 0xFFFFFFFFu, 0, 0};
+    LoadStats hs = {0, 0xFFFFFFFFu, 0, 0, 0};
     if (e == cudaSuccess) e = cudaMemcpy(dst, &hs, sizeof hs, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) {
         validate_rows_kernel<<<sms * 8, 256>>>(rp64, V, E, dst);
@@ -621,6 +640,7 @@ ag_status ag_graph_load_csr_ex(uint32_t V, uint64_t E, const uint64_t *row_ptr, 
     g->info.num_sms = sms;
     g->info.offset_bytes = g->offs32 ? 4 : 8;
     g->info.layout = g->layout;
+    g->info.max_weight = weights ? hs.max_w : 0;
     {   // L2 set-aside for the persisting status window (device-wide limit; never lowered)
         cudaDeviceProp pr;
         cudaGetDeviceProperties(&pr, device);

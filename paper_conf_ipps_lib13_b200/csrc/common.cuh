@@ -108,6 +108,7 @@ struct DevPolicy {
     uint32_t sample_every;
     uint32_t delta;
     uint32_t cta_group;   // resolved block-mapping group size (multiple of 32, <= BS)
+    uint32_t window;      // unordered SSSP deferral window (0 = off)
     uint32_t V;
     uint64_t E;
     uint32_t max_deg;     // inspector: maximum out-degree (tuned policy)

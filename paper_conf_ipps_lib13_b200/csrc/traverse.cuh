@@ -150,6 +150,15 @@ struct Ops {
                     vmin = min(vmin, t);
                 }
                 if (append_next) warp_append(q_next, qlen_next, !ex && (uint64_t)t >= hi, u);
+            } else if ((uint64_t)t >= hi) {
+                // unordered SSSP with a deferral window: a far vertex stays in the working set
+                // (re-added to the next frontier unless an improvement already did) and feeds the
+                // minimum that places the next window
+                ex = false;
+                vmin = min(vmin, t);
+                const uint32_t m = 1u << (u & 31);
+                const bool fresh = !(atomicOr(bm_next + (u >> 5), m) & m);
+                warp_append(q_next, qlen_next, fresh, u);
             }
         }
         if (ex) {
@@ -212,8 +221,8 @@ struct Ops {
                     if (fenced) __threadfence();
                     uint32_t ob = atomicOr(bm_next + (v >> 5), m);
                     nw = !(ob & m);                                    // ws.add(m), deduped  (l.9)
+                    vmin = min(vmin, (uint32_t)nd);
                     if constexpr (ORD == ORD_O) {
-                        vmin = min(vmin, (uint32_t)nd);
                         if (nw) dpend += 1;
                     }
                 }
@@ -459,9 +468,9 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, Tile
             if (ops.a.trace_edges) atomicAdd(&ctl->it_edges[slot], se);
         }
         if (sv) atomicAdd(&ctl->vexp, sv);
-        if (ALG == ALG_SSSP && ORD == ORD_O) {
+        if (ALG == ALG_SSSP) {
             if (mn != INF) atomicMin(&ctl->next_min[(slot + 1) % 3], mn);
-            if (sd) atomicAdd(&ctl->pend_count, (unsigned)sd);
+            if (ORD == ORD_O && sd) atomicAdd(&ctl->pend_count, (unsigned)sd);
         }
         if (ov) ctl->overflow = 1;
     }
@@ -785,9 +794,13 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             ctl->it_edges[rs] = 0;
         }
 
-        uint64_t hi = 0;
+        uint64_t hi = ~0ull;
         bool append = true;
         uint32_t qn = n;
+        if (ALG == ALG_SSSP && ROT && a.pol.window) {
+            const uint32_t lo = ld_relaxed(&ctl->next_min[slot]);
+            hi = (uint64_t)lo + a.pol.window;
+        }
         if (!ROT) {
             const uint32_t lo = ld_relaxed(&ctl->next_min[slot]);
             hi = (uint64_t)lo + a.pol.delta;

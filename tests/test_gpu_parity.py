@@ -108,6 +108,17 @@ def test_tiny_random_all_variants(seed, layout):
             check_sssp(g, G, s, p)
 
 
+@pytest.mark.parametrize("window", [0, 1, 7, 50, 300, 0xFFFFFFFF])
+def test_unordered_sssp_window(window):
+    """The deferral window reorders unordered SSSP but never changes the distances."""
+    for g in (aggen.config("C1"), aggen.with_weights(aggen.grid(60, 50), seed=9, wmax=100),
+              aggen.with_weights(aggen.er(5000, 20000, seed=4), seed=5, wmax=100)):
+        G = A.Graph.from_csr(g)
+        for s in aggen.sources(g, 2):
+            for m in (0, 1, 4):
+                check_sssp(g, G, s, pol(0, m, 2 if m else 0, sssp_window=window))
+
+
 @pytest.mark.parametrize("delta", [1, 7, 100, 1000])
 def test_ordered_sssp_delta(delta):
     g = aggen.config("C1")
