@@ -90,7 +90,10 @@ typedef struct {
     uint32_t sssp_window;    /* unordered SSSP: expand only frontier vertices with dist < min + window
                                 (others stay in the working set); 0 = off (plain Bellman-Ford rounds);
                                 AG_WINDOW_AUTO = tuned: off on skewed graphs, else 8 x max_weight / avg degree */
-    uint32_t reserved[3];    /* must be 0 */
+    uint32_t sssp_hub_window;/* unordered SSSP: vertices with out-degree >= 64 are expanded only when within
+                                this distance of the frontier minimum (re-expanding a hub re-scans its whole
+                                list); 0 = off; AG_WINDOW_AUTO = tuned: max(1, max_weight / 50) */
+    uint32_t reserved[2];    /* must be 0 */
 } ag_policy;
 
 typedef struct {

@@ -51,7 +51,7 @@ class Policy(ctypes.Structure):
                 ("workset", ctypes.c_uint32), ("kind", ctypes.c_uint32), ("t1_avg_degree", ctypes.c_uint32),
                 ("t2_ws", ctypes.c_uint64), ("t3_ppm", ctypes.c_uint32), ("sample_every", ctypes.c_uint32),
                 ("delta", ctypes.c_uint32), ("thread_tpb", ctypes.c_uint32), ("cta_group", ctypes.c_uint32),
-                ("sssp_window", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3)]
+                ("sssp_window", ctypes.c_uint32), ("sssp_hub_window", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 2)]
 
 
 class GraphInfo(ctypes.Structure):

@@ -259,6 +259,14 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
     } else {
         d.window = p.sssp_window;
     }
+    if (p.sssp_hub_window == AG_WINDOW_AUTO) {
+        // tuned: expand high-degree vertices only near the frontier minimum (R-MAT s22: edges
+        // inspected 2.75 E_r -> 1.15 E_r, 2.7 -> 1.9 ms; tools/sweep.py)
+        d.hub_window = (p.kind == AG_POLICY_TUNED && g.info.max_weight)
+                           ? (g.info.max_weight / 50 > 1 ? g.info.max_weight / 50 : 1u) : 0u;
+    } else {
+        d.hub_window = p.sssp_hub_window;
+    }
     d.V = g.V;
     d.E = g.E;
     d.max_deg = g.info.max_deg;
@@ -522,6 +530,7 @@ ag_status ag_policy_default(ag_policy *p, int device) {
     p->delta = 1;
     p->cta_group = 0;
     p->sssp_window = AG_WINDOW_AUTO;
+    p->sssp_hub_window = AG_WINDOW_AUTO;
     return AG_OK;
 }
 

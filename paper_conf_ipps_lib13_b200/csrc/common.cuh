@@ -66,6 +66,7 @@ enum { WS_BM = 1, WS_QU = 2 };
 #define AG_LONG_MIN 512   // hybrid mapping: lists this long go to aligned warp windows
 #endif
 constexpr uint32_t HUB_DEG = 2048;
+constexpr uint32_t HUBW_DEG = 64;   // SSSP hub-window degree threshold (measured on C1/C2/C4)
 constexpr uint32_t HUB_CHUNK = AG_HUBCHUNK;
 // Edges processed per thread per batch: loads of all EB edges are issued before any dependent use.
 constexpr int EB_MAX = (AG_EB_BFS > AG_EB_SSSP) ? AG_EB_BFS : AG_EB_SSSP;
@@ -109,6 +110,7 @@ struct DevPolicy {
     uint32_t delta;
     uint32_t cta_group;   // resolved block-mapping group size (multiple of 32, <= BS)
     uint32_t window;      // unordered SSSP deferral window (0 = off)
+    uint32_t hub_window;  // unordered SSSP deferral window for vertices of degree >= HUBW_DEG (0 = off)
     uint32_t V;
     uint64_t E;
     uint32_t max_deg;     // inspector: maximum out-degree (tuned policy)

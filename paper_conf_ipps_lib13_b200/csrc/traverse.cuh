@@ -98,6 +98,7 @@ struct Ops {
     const TravArgs<Off> &a;
     uint32_t it;
     uint64_t hi;            // SSSP ordered: exclusive bound lo + delta of the current bucket
+    uint64_t hub_hi = ~0ull;  // SSSP: deferral bound for high-degree vertices
     uint32_t *bm_next;      // next-frontier bitmap (SSSP ordered: the pending bitmap)
     uint32_t *q_next;
     unsigned *qlen_next;
@@ -150,7 +151,7 @@ struct Ops {
                     vmin = min(vmin, t);
                 }
                 if (append_next) warp_append(q_next, qlen_next, !ex && (uint64_t)t >= hi, u);
-            } else if ((uint64_t)t >= hi) {
+            } else if ((uint64_t)t >= hi || ((uint64_t)t >= hub_hi && (uint32_t)(a.rp[u + 1] - a.rp[u]) >= HUBW_DEG)) {
                 // unordered SSSP with a deferral window: a far vertex stays in the working set
                 // (re-added to the next frontier unless an improvement already did) and feeds the
                 // minimum that places the next window
@@ -830,6 +831,8 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
 
         Ops<ALG, ORD, Off> ops(a, it, hi, append);
         ops.wbuf = sm.wq[threadIdx.x >> 5];
+        if (ALG == ALG_SSSP && ROT && a.pol.hub_window)
+            ops.hub_hi = (uint64_t)ld_relaxed(&ctl->next_min[slot]) + a.pol.hub_window;
         const uint32_t *bmc = ROT ? a.bm[slot] : a.bm[0];
         const uint32_t *qc = a.q[slot];
         // queue tiles: BS entries for thread mapping (element per thread); for the cooperative

@@ -117,6 +117,7 @@ def test_unordered_sssp_window(window):
         for s in aggen.sources(g, 2):
             for m in (0, 1, 4):
                 check_sssp(g, G, s, pol(0, m, 2 if m else 0, sssp_window=window))
+                check_sssp(g, G, s, pol(0, m, 2 if m else 0, sssp_window=window, sssp_hub_window=1 + window % 5))
 
 
 @pytest.mark.parametrize("delta", [1, 7, 100, 1000])
