@@ -28,7 +28,7 @@ static_assert(LOG_BS > 0, "BS must be 128, 256, 512 or 1024");
 #define AG_MINB_BFS 5
 #endif
 #ifndef AG_MINB_SSSP
-#define AG_MINB_SSSP 8
+#define AG_MINB_SSSP 6
 #endif
 #ifndef AG_MINB_BFS_T
 #define AG_MINB_BFS_T AG_MINB_BFS
@@ -60,7 +60,7 @@ enum { WS_BM = 1, WS_QU = 2 };
 #define AG_QB 2           // hybrid mapping: aligned 16-byte pieces per thread per step (BFS)
 #endif
 #ifndef AG_QB_SSSP
-#define AG_QB_SSSP 1      //                                                  (SSSP)
+#define AG_QB_SSSP 2      //                                                  (SSSP)
 #endif
 #ifndef AG_LONG_MIN
 #define AG_LONG_MIN 512   // hybrid mapping: lists this long go to aligned warp windows

@@ -44,7 +44,7 @@ struct TravArgs {
     const uint32_t *inv;        //                caller id -> new id
     uint32_t *out_level;        // BFS outputs in caller ids (written by the final pass if relabelled)
     uint32_t *out_parent;
-    unsigned long long *P;      // SSSP packed state (V)
+    unsigned long long *P;      // SSSP packed state (V): (dist << 32) | parent, decided by 64-bit atomicMin
     uint32_t *vis;              // BFS ordered: visited bitmap
     uint32_t *bm[3];            // rotating frontier bitmaps (SSSP ordered: bm[0] = pending bitmap)
     uint32_t *q[3];             // rotating queues (capacity V)
@@ -177,9 +177,9 @@ struct Ops {
     // Status word of v, read before deciding to update.  Plain (L1-cacheable) load: a stale value is
     // always safe because levels/distances only decrease and visited bits are only set — a stale
     // read can only cause an extra atomic, never a missed update.
-    using St = typename std::conditional<ALG == ALG_SSSP, unsigned long long, uint32_t>::type;
+    using St = uint32_t;
     __device__ __forceinline__ St status(uint32_t v) const {
-        if constexpr (ALG == ALG_SSSP) return ld_keep(a.P + v, pol_keep);
+        if constexpr (ALG == ALG_SSSP) return (uint32_t)(ld_keep(a.P + v, pol_keep) >> 32);
         else return ld_keep(a.vis + (v >> 5), pol_keep);   // BFS: visited bit (level-synchronous: set <=> level <= current+1)
     }
 
@@ -216,7 +216,7 @@ struct Ops {
             const uint64_t nd = (uint64_t)uval + wt;                   // d = n.distance + w (Fig. 5 l.6)
             if (nd > MAX_FINITE) {
                 ovf = true;
-            } else if ((s >> 32) > nd) {                               // d < m.distance      (l.7)
+            } else if ((uint64_t)s > nd) {                             // d < m.distance      (l.7)
                 unsigned long long old = atomicMin(&a.P[v], (nd << 32) | u);
                 if ((old >> 32) > nd) {                                // m.distance = d      (l.8)
                     if (fenced) __threadfence();
