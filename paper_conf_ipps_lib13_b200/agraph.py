@@ -346,3 +346,35 @@ def _stats_out(st, tr):
     if tr is not None:
         res.trace_ws = tr[0][: st.trace_len]
     return res
+
+
+# ---------------------------------------------------------------------------------------------
+# device allocator hook (ag_set_allocator): route the library's device allocations through the
+# PyTorch caching allocator, so repeated graph loads reuse memory instead of cudaMalloc/cudaFree
+# ---------------------------------------------------------------------------------------------
+_ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p)
+_FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p)
+_alloc_refs = None
+
+
+def use_torch_allocator(enable: bool = True):
+    global _alloc_refs
+    L = lib()
+    L.ag_set_allocator.argtypes = [_ALLOC_T, _FREE_T, ctypes.c_void_p]
+    if not enable:
+        _check(L.ag_set_allocator(_ALLOC_T(0), _FREE_T(0), None))
+        _alloc_refs = None
+        return
+    import torch
+
+    def _alloc(nbytes, dev, stream, ctx):
+        try:
+            return torch.cuda.caching_allocator_alloc(int(nbytes), int(dev))
+        except Exception:
+            return 0
+
+    def _free(ptr, nbytes, dev, stream, ctx):
+        torch.cuda.caching_allocator_delete(int(ptr))
+
+    _alloc_refs = (_ALLOC_T(_alloc), _FREE_T(_free))
+    _check(L.ag_set_allocator(_alloc_refs[0], _alloc_refs[1], None))

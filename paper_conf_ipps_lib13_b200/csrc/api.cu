@@ -77,6 +77,33 @@ bool is_device_ptr(const void *p) {
     return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
 }
 
+// per-device attributes, queried once (cudaGetDeviceProperties is slow: milliseconds per call)
+struct DevAttrs {
+    bool valid = false;
+    int major = 0, minor = 0, sms = 0, persist_max = 0, window_max = 0;
+};
+static DevAttrs g_dev[64];
+static std::mutex g_dev_mu;
+
+const DevAttrs *device_attrs(int device) {
+    if (device < 0 || device >= 64) return nullptr;
+    std::lock_guard<std::mutex> lk(g_dev_mu);
+    DevAttrs &d = g_dev[device];
+    if (!d.valid) {
+        if (cudaDeviceGetAttribute(&d.major, cudaDevAttrComputeCapabilityMajor, device) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        cudaDeviceGetAttribute(&d.minor, cudaDevAttrComputeCapabilityMinor, device);
+        cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, device);
+        cudaDeviceGetAttribute(&d.persist_max, cudaDevAttrMaxPersistingL2CacheSize, device);
+        cudaDeviceGetAttribute(&d.window_max, cudaDevAttrMaxAccessPolicyWindowSize, device);
+        cudaGetLastError();
+        d.valid = true;
+    }
+    return &d;
+}
+
 ag_status check_device(int device, int *num_sms) {
     int n = 0;
     cudaError_t e = cudaGetDeviceCount(&n);
@@ -85,12 +112,12 @@ ag_status check_device(int device, int *num_sms) {
         return set_error(AG_ERR_NO_DEVICE, "no CUDA device available");
     }
     if (device < 0 || device >= n) return set_error(AG_ERR_INVALID_ARG, "device %d out of range [0,%d)", device, n);
-    cudaDeviceProp pr;
-    if ((e = cudaGetDeviceProperties(&pr, device)) != cudaSuccess) return cuda_status(e, "cudaGetDeviceProperties");
-    if (pr.major != 10 || pr.minor != 0)
+    const DevAttrs *d = device_attrs(device);
+    if (!d) return set_error(AG_ERR_CUDA, "cannot query device %d", device);
+    if (d->major != 10 || d->minor != 0)
         return set_error(AG_ERR_NO_DEVICE, "device %d is sm_%d%d; libagraph is built for sm_100a only", device,
-                         pr.major, pr.minor);
-    if (num_sms) *num_sms = pr.multiProcessorCount;
+                         d->major, d->minor);
+    if (num_sms) *num_sms = d->sms;
     return AG_OK;
 }
 }  // namespace ag
@@ -650,17 +677,16 @@ ag_status ag_graph_load_csr_ex(uint32_t V, uint64_t E, const uint64_t *row_ptr, 
     g->info.offset_bytes = g->offs32 ? 4 : 8;
     g->info.layout = g->layout;
     g->info.max_weight = weights ? hs.max_w : 0;
-    {   // L2 set-aside for the persisting status window (device-wide limit; never lowered)
-        cudaDeviceProp pr;
-        cudaGetDeviceProperties(&pr, device);
-        size_t want = (size_t)V * 8;
-        if (want > (size_t)pr.persistingL2CacheMaxSize) want = (size_t)pr.persistingL2CacheMaxSize;
+    {   // L2 set-aside for the persisting status window (device-wide limit, set once to the maximum)
+        const DevAttrs *da = device_attrs(device);
         size_t cur = 0;
         cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
-        if (want > cur) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want);
-        cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+        if (da && cur < (size_t)da->persist_max) {
+            cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)da->persist_max);
+            cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+        }
         g->persist_bytes = cur;
-        g->max_window = (size_t)pr.accessPolicyMaxWindowSize;
+        g->max_window = da ? (size_t)da->window_max : 0;
         cudaGetLastError();
     }
     *out = g;

@@ -65,7 +65,10 @@ enum { WS_BM = 1, WS_QU = 2 };
 #ifndef AG_LONG_MIN
 #define AG_LONG_MIN 512   // hybrid mapping: lists this long go to aligned warp windows
 #endif
-constexpr uint32_t HUB_DEG = 2048;
+#ifndef AG_HUBDEG
+#define AG_HUBDEG 2048
+#endif
+constexpr uint32_t HUB_DEG = AG_HUBDEG;
 constexpr uint32_t HUBW_DEG = 64;   // SSSP hub-window degree threshold (measured on C1/C2/C4)
 constexpr uint32_t HUB_CHUNK = AG_HUBCHUNK;
 // Edges processed per thread per batch: loads of all EB edges are issued before any dependent use.

@@ -281,3 +281,25 @@ def test_full_size_configs(cfg):
             check_bfs(g, G, s, pol(1))
     if cfg in ("C3", "C3p"):
         check_sssp(g, G, srcs[-1], pol(1, delta=1 if cfg == "C3p" else 64))
+
+
+def test_torch_allocator_hook():
+    """ag_set_allocator routes every device buffer through the PyTorch caching allocator."""
+    import torch
+    g = aggen.config("C1")
+    s = int(aggen.sources(g, 1)[0])
+    lv, _ = oracle.bfs(g, s)
+    d, _ = oracle.dijkstra(g, s)
+    A.use_torch_allocator(True)
+    try:
+        before = torch.cuda.memory_allocated()
+        G = A.Graph.from_csr(g)
+        out, _, _ = G.bfs(s)
+        assert np.array_equal(out, lv)
+        out, _, _ = G.sssp(s)
+        assert np.array_equal(out, d)
+        assert torch.cuda.memory_allocated() > before      # the library's buffers live in torch's pool
+        G.free()
+        assert torch.cuda.memory_allocated() == before
+    finally:
+        A.use_torch_allocator(False)
