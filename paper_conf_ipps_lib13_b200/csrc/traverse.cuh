@@ -233,6 +233,86 @@ struct Ops {
         return nw;
     }
 
+    // The updates of NB edges with their atomics phased: (1) candidates from the status words,
+    // (2) every claiming atomic of the batch issued back to back, (3) results resolved.  A thread with
+    // several discoveries then waits for one atomic round trip, not several in a row.  Same semantics
+    // as NB calls of update(); returns bit j set if v[j] newly entered the next working set.
+    template <int NB>
+    __device__ __forceinline__ uint32_t update_batch(const uint32_t (&u)[NB], const uint32_t (&uv)[NB],
+                                                     const uint32_t (&v)[NB], const uint32_t (&wt)[NB],
+                                                     const St (&st)[NB], const bool (&ok)[NB]) {
+        uint32_t nwm = 0;
+        if constexpr (ALG == ALG_BFS) {
+            uint32_t r[NB];
+            uint32_t cm = 0;   // bit j: an atomic was issued for edge j
+#pragma unroll
+            for (int j = 0; j < NB; ++j) {
+                const uint32_t m = 1u << (v[j] & 31);
+                r[j] = 0u;
+                if (ok[j] && !(st[j] & m)) {                           // m.level == INF / > level
+                    cm |= 1u << j;
+                    if constexpr (ORD == ORD_O) r[j] = atomicOr(a.vis + (v[j] >> 5), m);  // claim
+                    else r[j] = atomicMin(&a.level[v[j]], uv[j] + 1);
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < NB; ++j) {
+                const uint32_t m = 1u << (v[j] & 31);
+                const uint32_t nl = uv[j] + 1;
+                const bool won = ((cm >> j) & 1u) && ((ORD == ORD_O) ? !(r[j] & m) : (r[j] > nl));
+                if (won) {
+                    if constexpr (ORD == ORD_O) {
+                        a.level[v[j]] = nl;                            // m.level = level    (l.9)
+                        red_or(a.bm[(it + 1) % 3] + (v[j] >> 5), m);   // update vector      (l.10)
+                    } else {
+                        red_or(a.vis + (v[j] >> 5), m);
+                        red_or(bm_next + (v[j] >> 5), m);
+                    }
+                    if (a.parent) a.parent[v[j]] = u[j];
+                    nwm |= 1u << j;
+                }
+            }
+        } else {
+            unsigned long long r[NB];
+            uint64_t nd[NB];
+            uint32_t cm = 0;   // bit j: atomicMin issued for edge j
+#pragma unroll
+            for (int j = 0; j < NB; ++j) {
+                nd[j] = (uint64_t)uv[j] + wt[j];                        // d = n.distance + w (l.6)
+                r[j] = 0ull;
+                if (ok[j]) {
+                    if (nd[j] > MAX_FINITE) {
+                        ovf = true;
+                    } else if ((uint64_t)st[j] > nd[j]) {               // d < m.distance      (l.7)
+                        cm |= 1u << j;
+                        r[j] = atomicMin(&a.P[v[j]], (nd[j] << 32) | u[j]);
+                    }
+                }
+            }
+            uint32_t ob[NB];
+            uint32_t im = 0;   // bit j: we lowered m.distance
+#pragma unroll
+            for (int j = 0; j < NB; ++j) {
+                ob[j] = 0u;
+                if (((cm >> j) & 1u) && (r[j] >> 32) > nd[j]) {         // m.distance = d      (l.8)
+                    if (fenced) __threadfence();
+                    im |= 1u << j;
+                    ob[j] = atomicOr(bm_next + (v[j] >> 5), 1u << (v[j] & 31));
+                    vmin = min(vmin, (uint32_t)nd[j]);
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < NB; ++j) {
+                const bool nw = ((im >> j) & 1u) && !(ob[j] & (1u << (v[j] & 31)));  // ws.add(m) (l.9)
+                if (nw) {
+                    if constexpr (ORD == ORD_O) dpend += 1;
+                    if (ORD == ORD_U || append_next) nwm |= 1u << j;
+                }
+            }
+        }
+        return nwm;
+    }
+
     // NB independent edges: all CSR loads first, then all status loads, then the updates, so NB
     // memory requests per phase are in flight per thread (the per-edge chain col -> status -> atomic
     // is latency-bound otherwise).  New working-set elements are appended either warp-aggregated to
@@ -283,9 +363,7 @@ struct Ops {
         }
 #endif
         if constexpr (STAGED) {
-            uint32_t nwm = 0;   // bit j: v[j] entered the next working set
-#pragma unroll
-            for (int j = 0; j < NB; ++j) nwm |= update(u[j], uv[j], v[j], wt[j], st[j], ok[j]) ? (1u << j) : 0u;
+            const uint32_t nwm = update_batch<NB>(u, uv, v, wt, st, ok);  // bit j: v[j] entered the next WS
             if (__any_sync(0xffffffffu, nwm != 0)) {   // rare on the big levels: skip the ballots otherwise
 #pragma unroll
                 for (int j = 0; j < NB; ++j) {
@@ -298,11 +376,9 @@ struct Ops {
                 if (wfill >= 32) warp_flush(false);
             }
         } else {
+            const uint32_t nwm = update_batch<NB>(u, uv, v, wt, st, ok);
 #pragma unroll
-            for (int j = 0; j < NB; ++j) {
-                bool nw = update(u[j], uv[j], v[j], wt[j], st[j], ok[j]);
-                warp_append(q_next, qlen_next, nw, v[j]);
-            }
+            for (int j = 0; j < NB; ++j) warp_append(q_next, qlen_next, (nwm >> j) & 1u, v[j]);
         }
     }
 
