@@ -616,7 +616,6 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<O
                 tk[0] = u;
                 tk[1] = uval;
                 tk[2] = k;
-                __threadfence();
                 st_release(tk + 3, tag);
             } else {
                 a.ctl->aborted = 2;
@@ -697,15 +696,17 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, TileSmem<Off
             const uint32_t t = claimed;
             uint32_t status = 0;  // 0 = done, 1 = ready
             for (;;) {
-                uint32_t tail = ld_acquire(&ctl->hub_tail[slot]);
+                uint32_t tail = ld_relaxed(&ctl->hub_tail[slot]);
                 if (t < tail) {
                     if (t >= a.hub_cap) { status = 0; break; }
-                    while (ld_acquire(a.hub + 4ull * t + 3) != tag) __nanosleep(32);
+                    while (ld_relaxed(a.hub + 4ull * t + 3) != tag) __nanosleep(32);
+                    (void)ld_acquire(a.hub + 4ull * t + 3);
                     status = 1;
                     break;
                 }
-                if (ld_acquire(&ctl->stage_done[slot]) == a.nblocks) {
-                    if (t < ld_acquire(&ctl->hub_tail[slot])) continue;
+                if (ld_relaxed(&ctl->stage_done[slot]) == a.nblocks) {
+                    (void)ld_acquire(&ctl->stage_done[slot]);
+                    if (t < ld_relaxed(&ctl->hub_tail[slot])) continue;
                     status = 0;
                     break;
                 }
