@@ -48,7 +48,7 @@ def main():
     if nsass:
         rows = list(csv.reader(io.StringIO(ncu([rep, "--page", "source", "--csv", "--print-source=sass"]))))
         hdr = rows[1]
-        data = rows[2:]
+        data = [r for r in rows[2:] if len(r) == len(hdr) and r[hdr.index("Warp Stall Sampling (All Samples)")].replace('.', '', 1).isdigit()]
         iss = hdr.index("Warp Stall Sampling (All Samples)")
         isrc = hdr.index("Source")
         iex = hdr.index("Instructions Executed")
