@@ -237,7 +237,10 @@ static ag_status ensure_scratch(ag_graph_s *g, bool sssp) {
     for (int i = 0; i < 3; ++i) { ALLOC(g->d_bm[i], nw * 4 + 128); }
     for (int i = 0; i < 3; ++i) { ALLOC(g->d_q[i], V * 4 + 128); }
     ALLOC(g->d_vis, nw * 4 + 128);
-    ALLOC(g->d_hub, (size_t)g->hub_cap * 16);
+    if (!g->d_hub) {   // hub-task ring: every slot 0 (= empty) between iterations
+        ALLOC(g->d_hub, (size_t)g->hub_cap * 8);
+        cudaMemset(g->d_hub, 0, (size_t)g->hub_cap * 8);
+    }
     ALLOC(g->d_acc, 64);
     if (sssp) { ALLOC(g->d_P, V * 8 + 128); }
 #undef ALLOC
@@ -512,6 +515,18 @@ uint32_t ag_abi_version(void) { return AG_ABI_VERSION; }
 uint64_t ag_kernel_launches(void) { return g_launches.load(); }
 const char *ag_last_error(void) { return g_last_error.c_str(); }
 
+// diagnostic builds (-DAG_PROF) only: copy the per-(iteration, CTA) timestamps to host memory
+int ag_debug_prof(void *host, size_t bytes) {
+#ifdef AG_PROF
+    size_t n = sizeof(ag::g_prof) < bytes ? sizeof(ag::g_prof) : bytes;
+    return cudaMemcpyFromSymbol(host, ag::g_prof, n) == cudaSuccess ? (int)ag::PROF_CTA : -1;
+#else
+    (void)host;
+    (void)bytes;
+    return -1;
+#endif
+}
+
 const char *ag_status_string(ag_status s) {
     switch (s) {
         case AG_OK: return "AG_OK";
@@ -711,7 +726,7 @@ ag_status ag_graph_free(ag_graph g) {
     dev_free(g->d_ctl, sizeof(Ctl), g->device);
     for (int i = 0; i < 3; ++i) { dev_free(g->d_bm[i], nw * 4 + 128, g->device); dev_free(g->d_q[i], V * 4 + 128, g->device); }
     dev_free(g->d_vis, nw * 4 + 128, g->device);
-    dev_free(g->d_hub, (size_t)g->hub_cap * 16, g->device);
+    dev_free(g->d_hub, (size_t)g->hub_cap * 8, g->device);
     dev_free(g->d_acc, 64, g->device);
     dev_free(g->d_P, V * 8 + 128, g->device);
     dev_free(g->d_out_tmp, g->out_tmp_bytes, g->device);
@@ -738,7 +753,10 @@ ag_status ag_graph_check(ag_graph g) {
     Ctl c;
     e = cudaMemcpy(&c, g->d_ctl, sizeof c, cudaMemcpyDeviceToHost);
     if (e != cudaSuccess) return cuda_status(e, "ctl");
-    if (c.aborted) return set_error(AG_ERR_CUDA, "traversal aborted (code %u)", c.aborted);
+    if (c.aborted) {
+        if (g->d_hub) cudaMemset(g->d_hub, 0, (size_t)g->hub_cap * 8);   // the ring may hold unconsumed tasks
+        return set_error(AG_ERR_CUDA, "traversal aborted (code %u)", c.aborted);
+    }
     if (g->last_alg == ALG_SSSP && c.overflow) {
         unsigned *flag = (unsigned *)g->d_acc;
         cudaMemset(flag, 0, 4);

@@ -65,6 +65,9 @@ enum { WS_BM = 1, WS_QU = 2 };
 #ifndef AG_LONG_MIN
 #define AG_LONG_MIN 512   // hybrid mapping: lists this long go to aligned warp windows
 #endif
+#ifndef AG_WARPH
+#define AG_WARPH 0        // hybrid mapping tiles scheduled per warp (1) or per CTA (0)
+#endif
 #ifndef AG_HUBDEG
 #define AG_HUBDEG 2048
 #endif
@@ -162,6 +165,9 @@ __device__ __forceinline__ unsigned ld_relaxed(const unsigned *p) {
     unsigned v;
     asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
+}
+__device__ __forceinline__ void st_relaxed64(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 __device__ __forceinline__ unsigned long long ld_relaxed64(const unsigned long long *p) {
     unsigned long long v;

@@ -205,7 +205,6 @@ __global__ void __launch_bounds__(BS, AG_MINB_BFS) dist_level_kernel(const TravA
     uint32_t tile_n = (qn + 2 * a.nblocks - 1) / (2 * a.nblocks);
     tile_n = tile_n < 1u ? 1u : (tile_n > (uint32_t)BS ? (uint32_t)BS : tile_n);
     const uint32_t ntiles = (qn + tile_n - 1) / tile_n;
-    const uint32_t tag = a.epoch * 0x9E3779B1u + L + 1;
     uint32_t t = blockIdx.x;
     int par = 0;
     while (t < ntiles) {
@@ -213,11 +212,11 @@ __global__ void __launch_bounds__(BS, AG_MINB_BFS) dist_level_kernel(const TravA
         const uint32_t i = t * tile_n + threadIdx.x;
         const bool valid = threadIdx.x < tile_n && i < qn;
         const uint32_t u = valid ? a.q[0][i] : 0u;
-        if (__syncthreads_or(valid)) process_tile<true>(ops, sm, MAP_H, valid, u, 32u, a.has_hubs != 0, slot, tag);
+        if (__syncthreads_or(valid)) process_tile<true>(ops, sm, MAP_H, valid, u, 32u, a.has_hubs != 0, slot);
         t = sm.tnext[par];
         par ^= 1;
     }
-    if (a.has_hubs) drain_hubs(ops, sm, slot, tag);
+    if (a.has_hubs) drain_hubs(ops, sm, slot);
     ops.warp_flush(true);
     block_reduce_flush(ops, sm, ctl, slot);
 }
@@ -256,7 +255,10 @@ ag_status dist_scratch(ag_graph_s *g) {
     if (!g->d_q[0] && (s = dev_alloc((void **)&g->d_q[0], V * 4 + 128, g->device)) != AG_OK) return s;
     if (!g->d_q[1] && (s = dev_alloc((void **)&g->d_q[1], V * 4 + 128, g->device)) != AG_OK) return s;
     if (!g->d_vis && (s = dev_alloc((void **)&g->d_vis, gw * 4 + 128, g->device)) != AG_OK) return s;
-    if (!g->d_hub && (s = dev_alloc((void **)&g->d_hub, (size_t)g->hub_cap * 16, g->device)) != AG_OK) return s;
+    if (!g->d_hub) {
+        if ((s = dev_alloc((void **)&g->d_hub, (size_t)g->hub_cap * 8, g->device)) != AG_OK) return s;
+        cudaMemset(g->d_hub, 0, (size_t)g->hub_cap * 8);
+    }
     if (!g->d_level && (s = dev_alloc((void **)&g->d_level, V * 4 + 128, g->device)) != AG_OK) return s;
     if (!g->d_acc && (s = dev_alloc(&g->d_acc, 64, g->device)) != AG_OK) return s;
     return AG_OK;

@@ -41,7 +41,7 @@ struct ag_graph_s {
     uint32_t *d_bm[3] = {nullptr, nullptr, nullptr};
     uint32_t *d_q[3] = {nullptr, nullptr, nullptr};
     uint32_t *d_vis = nullptr;
-    uint32_t *d_hub = nullptr;
+    unsigned long long *d_hub = nullptr;   // hub-task ring (self-contained 64-bit task words)
     uint32_t hub_cap = 0;
     unsigned long long *d_P = nullptr;
     void *d_acc = nullptr;

@@ -31,6 +31,17 @@
 
 namespace ag {
 
+#ifdef AG_PROF
+// diagnostic build only: per (iteration, CTA) timestamps — iteration start, tile loop done, hub drain
+// done — read back with ag_debug_prof() (tools/prof_iters.py)
+constexpr int PROF_IT = 64, PROF_CTA = 2048;
+__device__ unsigned long long g_prof[PROF_IT][PROF_CTA][3];
+#define AG_PROF_MARK(it, k) \
+    if (threadIdx.x == 0 && (it) < PROF_IT && blockIdx.x < PROF_CTA) g_prof[it][blockIdx.x][k] = globaltimer_ns()
+#else
+#define AG_PROF_MARK(it, k)
+#endif
+
 template <typename Off>
 struct TravArgs {
     const Off *rp;
@@ -48,7 +59,7 @@ struct TravArgs {
     uint32_t *vis;              // BFS ordered: visited bitmap
     uint32_t *bm[3];            // rotating frontier bitmaps (SSSP ordered: bm[0] = pending bitmap)
     uint32_t *q[3];             // rotating queues (capacity V)
-    uint32_t *hub;              // hybrid hub-chunk tasks, 4 words each
+    unsigned long long *hub;    // hybrid hub-chunk task ring (one 64-bit word per task, 0 = empty)
     uint32_t hub_cap;
     Ctl *ctl;
     uint32_t *dist_out;         // SSSP outputs (V) — may alias nothing
@@ -83,9 +94,10 @@ struct __align__(16) TileSmem {
     unsigned long long red64[2][WARPS_PER_CTA];
     uint32_t red32[2][WARPS_PER_CTA];
     int redi[WARPS_PER_CTA];
+    uint32_t wsc[WARPS_PER_CTA][32];   // warp-tile piece scan (warp-scheduled hybrid mapping)
     uint32_t tnext[2];
     uint32_t bcast;
-    uint32_t htask[2][4];   // hub-drain task slots (u, uval, chunk, status)
+    unsigned long long htask[2];   // hub-drain task slots (task word, 0 = drained)
 };
 
 // ------------------------------------------------------------------------------------------------
@@ -237,20 +249,37 @@ struct Ops {
     // (2) every claiming atomic of the batch issued back to back, (3) results resolved.  A thread with
     // several discoveries then waits for one atomic round trip, not several in a row.  Same semantics
     // as NB calls of update(); returns bit j set if v[j] newly entered the next working set.
-    template <int NB>
+    template <int NB, bool CONV = false>
     __device__ __forceinline__ uint32_t update_batch(const uint32_t (&u)[NB], const uint32_t (&uv)[NB],
                                                      const uint32_t (&v)[NB], const uint32_t (&wt)[NB],
                                                      const St (&st)[NB], const bool (&ok)[NB]) {
+        // (1) candidates from the (possibly stale) status words; CONV (all 32 lanes converged): a warp
+        // with no candidate at all skips the atomic and resolution code (the common case on big levels)
+        uint32_t cm = 0;   // bit j: an atomic is issued for edge j
+        uint64_t nd[NB];
+#pragma unroll
+        for (int j = 0; j < NB; ++j) {
+            if constexpr (ALG == ALG_BFS) {
+                nd[j] = 0;
+                if (ok[j] && !((st[j] >> (v[j] & 31)) & 1u)) cm |= 1u << j;   // m.level == INF / > level
+            } else {
+                nd[j] = (uint64_t)uv[j] + wt[j];                                // d = n.distance + w (l.6)
+                if (ok[j]) {
+                    if (nd[j] > MAX_FINITE) ovf = true;
+                    else if ((uint64_t)st[j] > nd[j]) cm |= 1u << j;            // d < m.distance      (l.7)
+                }
+            }
+        }
+        if (CONV && !__any_sync(0xffffffffu, cm != 0)) return 0u;
         uint32_t nwm = 0;
         if constexpr (ALG == ALG_BFS) {
+            // (2) every claiming atomic of the batch issued back to back, (3) results resolved
             uint32_t r[NB];
-            uint32_t cm = 0;   // bit j: an atomic was issued for edge j
 #pragma unroll
             for (int j = 0; j < NB; ++j) {
                 const uint32_t m = 1u << (v[j] & 31);
                 r[j] = 0u;
-                if (ok[j] && !(st[j] & m)) {                           // m.level == INF / > level
-                    cm |= 1u << j;
+                if ((cm >> j) & 1u) {
                     if constexpr (ORD == ORD_O) r[j] = atomicOr(a.vis + (v[j] >> 5), m);  // claim
                     else r[j] = atomicMin(&a.level[v[j]], uv[j] + 1);
                 }
@@ -274,20 +303,10 @@ struct Ops {
             }
         } else {
             unsigned long long r[NB];
-            uint64_t nd[NB];
-            uint32_t cm = 0;   // bit j: atomicMin issued for edge j
 #pragma unroll
             for (int j = 0; j < NB; ++j) {
-                nd[j] = (uint64_t)uv[j] + wt[j];                        // d = n.distance + w (l.6)
                 r[j] = 0ull;
-                if (ok[j]) {
-                    if (nd[j] > MAX_FINITE) {
-                        ovf = true;
-                    } else if ((uint64_t)st[j] > nd[j]) {               // d < m.distance      (l.7)
-                        cm |= 1u << j;
-                        r[j] = atomicMin(&a.P[v[j]], (nd[j] << 32) | u[j]);
-                    }
-                }
+                if ((cm >> j) & 1u) r[j] = atomicMin(&a.P[v[j]], (nd[j] << 32) | u[j]);
             }
             uint32_t ob[NB];
             uint32_t im = 0;   // bit j: we lowered m.distance
@@ -363,7 +382,7 @@ struct Ops {
         }
 #endif
         if constexpr (STAGED) {
-            const uint32_t nwm = update_batch<NB>(u, uv, v, wt, st, ok);  // bit j: v[j] entered the next WS
+            const uint32_t nwm = update_batch<NB, true>(u, uv, v, wt, st, ok);  // bit j: v[j] entered the next WS
             if (__any_sync(0xffffffffu, nwm != 0)) {   // rare on the big levels: skip the ballots otherwise
 #pragma unroll
                 for (int j = 0; j < NB; ++j) {
@@ -559,8 +578,7 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, Tile
 // ------------------------------------------------------------------------------------------------
 template <bool TUNED, int ALG, int ORD, typename Off>
 __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<Off> &sm, uint32_t map,
-                                             bool valid, uint32_t u, uint32_t group, bool hubs, uint32_t slot,
-                                             uint32_t tag) {
+                                             bool valid, uint32_t u, uint32_t group, bool hubs, uint32_t slot) {
     const TravArgs<Off> &a = ops.a;
     Off beg = 0;
     uint32_t deg = 0, uval = 0;
@@ -609,17 +627,13 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<O
         uint32_t base = atomicAdd(&a.ctl->hub_tail[slot], nch);
         // hub_cap >= E/HUB_CHUNK + E/HUB_DEG + 16 covers any frontier (each vertex is at most once
         // per iteration in it); the guard only protects memory.
+        // a task is ONE self-contained 64-bit word (u << 32 | chunk << 1 | 1), published with a single
+        // relaxed store: the consumer needs no acquire (which would invalidate its L1) and clears the
+        // slot after reading it, so a nonzero word is always a task of the current iteration
         for (uint32_t k = 0; k < nch; ++k) {
             uint32_t idx = base + k;
-            if (idx < a.hub_cap) {
-                uint32_t *tk = a.hub + 4ull * idx;
-                tk[0] = u;
-                tk[1] = uval;
-                tk[2] = k;
-                st_release(tk + 3, tag);
-            } else {
-                a.ctl->aborted = 2;
-            }
+            if (idx < a.hub_cap) st_relaxed64(a.hub + idx, ((unsigned long long)u << 32) | ((unsigned long long)k << 1) | 1ull);
+            else a.ctl->aborted = 2;
         }
     }
     // every (non-hub) adjacency list is cut into aligned 16-byte pieces (QE entries each: 4 col ids for
@@ -675,56 +689,127 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<O
     // no trailing barrier: the next tile's __syncthreads_or orders the reuse of the tile arrays
 }
 
-// drain the hub-chunk tasks of this iteration (hybrid mapping)
+// Warp-scheduled hybrid mapping (AG_WARPH): the same load-balanced gather over aligned 16-byte
+// pieces as process_tile, but each warp claims its own tiles of <= 32 working-set elements (one
+// atomic per warp tile), scans its lanes' piece counts with shuffles and finds piece owners with a
+// 5-step search over its own 32 scan entries: no CTA barrier in the expansion, so a warp stalled on
+// gathers never holds up the other warps of its CTA.  Hub lists still go to the CTA-level drain.
 template <int ALG, int ORD, typename Off>
-__device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, TileSmem<Off> &sm, uint32_t slot,
-                                           uint32_t tag) {
+__device__ __forceinline__ void process_warp_tile(Ops<ALG, ORD, Off> &ops, TileSmem<Off> &sm, bool valid, uint32_t u,
+                                                  bool hubs, uint32_t slot) {
+    const TravArgs<Off> &a = ops.a;
+    Off beg = 0;
+    uint32_t deg = 0, uval = 0;
+    const bool ex = valid && ops.gate(u, beg, deg, uval);
+    if (!ex) deg = 0;
+    const uint32_t tid = threadIdx.x, lane = lane_id(), wid = tid >> 5;
+    const bool is_hub = hubs && deg >= HUB_DEG;
+    if (is_hub) {
+        const uint32_t nch = (deg + HUB_CHUNK - 1) / HUB_CHUNK;
+        uint32_t base = atomicAdd(&a.ctl->hub_tail[slot], nch);
+        for (uint32_t k = 0; k < nch; ++k) {
+            uint32_t idx = base + k;
+            if (idx < a.hub_cap) st_relaxed64(a.hub + idx, ((unsigned long long)u << 32) | ((unsigned long long)k << 1) | 1ull);
+            else a.ctl->aborted = 2;
+        }
+    }
+    constexpr uint32_t QE = Ops<ALG, ORD, Off>::QE;
+    constexpr int QB = Ops<ALG, ORD, Off>::QB;
+    const uint32_t d = is_hub ? 0u : deg;
+    const uint32_t np = d ? (uint32_t)((beg + d + QE - 1) / QE - beg / QE) : 0u;
+    uint32_t x = np;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        uint32_t xo = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= (unsigned)o) x += xo;
+    }
+    const uint32_t NP = __shfl_sync(0xffffffffu, x, 31);
+    if (NP == 0) return;
+    __syncwarp();   // the previous warp tile's readers are done with the per-warp arrays
+    sm.u[tid] = u;
+    sm.uval[tid] = uval;
+    sm.beg[tid] = beg;
+    sm.deg[tid] = d;
+    uint32_t *sc = sm.wsc[wid];
+    sc[lane] = x - np;
+    __syncwarp();
+    const uint32_t w0 = wid * 32;
+    for (uint32_t base = 0; base < NP; base += QB * 32) {
+        uint32_t pu[QB], pv[QB];
+        Off pq[QB], plo[QB], phi[QB];
+        bool pok[QB];
+#pragma unroll
+        for (int j = 0; j < QB; ++j) {
+            const uint32_t p = base + j * 32 + lane;
+            pok[j] = p < NP;
+            uint32_t lo = 0;   // owner: the largest lane i with scan[i] <= p
+#pragma unroll
+            for (int step = 16; step > 0; step >>= 1)
+                if (sc[lo + step] <= p) lo += step;
+            const uint32_t o = w0 + lo;
+            pu[j] = sm.u[o];
+            pv[j] = sm.uval[o];
+            const Off bo = sm.beg[o];
+            plo[j] = bo;
+            phi[j] = bo + sm.deg[o];
+            pq[j] = bo / QE + (p - sc[lo]);   // aligned piece index
+        }
+        ops.template pieces<QB>(pu, pv, pq, plo, phi, pok);
+    }
+}
+
+// Wait for hub task t of this iteration: its word, or 0 once the producers are all done and t is
+// past the final tail (thread 0 only).
+template <typename Off>
+__device__ __forceinline__ unsigned long long hub_wait(const TravArgs<Off> &a, uint32_t t, uint32_t slot) {
+    Ctl *ctl = a.ctl;
+    if (t >= a.hub_cap) return 0ull;   // overflow (flagged by the producer)
+    for (;;) {
+        const unsigned long long w = ld_relaxed64(a.hub + t);
+        if (w) return w;
+        if (t < ld_relaxed(&ctl->hub_tail[slot])) {   // reserved, not yet written
+            __nanosleep(32);
+            continue;
+        }
+        if (ld_relaxed(&ctl->stage_done[slot]) == a.nblocks) {
+            (void)ld_acquire(&ctl->stage_done[slot]);   // every producer's tail reservation is visible
+            if (t < ld_relaxed(&ctl->hub_tail[slot])) continue;
+            return 0ull;
+        }
+        __nanosleep(64);
+    }
+}
+
+// drain the hub-chunk tasks of this iteration (hybrid mapping).  Thread 0 runs two claims ahead and
+// loads the next task word before the CTA expands the current one, so in steady state the claim and
+// fetch latency hides behind the expansion; tasks reach the CTA through two shared-memory slots.
+template <int ALG, int ORD, typename Off>
+__device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, TileSmem<Off> &sm, uint32_t slot) {
     const TravArgs<Off> &a = ops.a;
     Ctl *ctl = a.ctl;
     __syncthreads();
+    uint32_t c1 = 0, c2 = 0;          // claimed task indices: next, and the one after
+    unsigned long long pre = 0ull;    // prefetched word of task c1
     if (threadIdx.x == 0) {
         __threadfence();
         atomicAdd(&ctl->stage_done[slot], 1u);
+        const uint32_t c0 = atomicAdd(&ctl->hub_head[slot], 1u);
+        c1 = atomicAdd(&ctl->hub_head[slot], 1u);
+        const unsigned long long w = hub_wait(a, c0, slot);
+        if (w) {
+            a.hub[c0] = 0ull;
+            pre = c1 < a.hub_cap ? ld_relaxed64(a.hub + c1) : 0ull;
+            c2 = atomicAdd(&ctl->hub_head[slot], 1u);
+        }
+        sm.htask[0] = w;
     }
-    // the leader claims task indices one ahead (the claim's round trip overlaps the previous task);
-    // tasks are handed to the CTA through two shared-memory slots, one barrier per task
-    uint32_t claimed = 0;
-    if (threadIdx.x == 0) claimed = atomicAdd(&ctl->hub_head[slot], 1u);
+    __syncthreads();
     int par = 0;
     for (;;) {
-        if (threadIdx.x == 0) {
-            const uint32_t t = claimed;
-            uint32_t status = 0;  // 0 = done, 1 = ready
-            for (;;) {
-                uint32_t tail = ld_relaxed(&ctl->hub_tail[slot]);
-                if (t < tail) {
-                    if (t >= a.hub_cap) { status = 0; break; }
-                    while (ld_relaxed(a.hub + 4ull * t + 3) != tag) __nanosleep(32);
-                    (void)ld_acquire(a.hub + 4ull * t + 3);
-                    status = 1;
-                    break;
-                }
-                if (ld_relaxed(&ctl->stage_done[slot]) == a.nblocks) {
-                    (void)ld_acquire(&ctl->stage_done[slot]);
-                    if (t < ld_relaxed(&ctl->hub_tail[slot])) continue;
-                    status = 0;
-                    break;
-                }
-                __nanosleep(64);
-            }
-            if (status) {
-                const uint32_t *tk = a.hub + 4ull * t;
-                sm.htask[par][0] = tk[0];
-                sm.htask[par][1] = tk[1];
-                sm.htask[par][2] = tk[2];
-                claimed = atomicAdd(&ctl->hub_head[slot], 1u);   // prefetch the next claim
-            }
-            sm.htask[par][3] = status;
-        }
-        __syncthreads();
-        if (!sm.htask[par][3]) break;
-        const uint32_t u = sm.htask[par][0], uval = sm.htask[par][1], k = sm.htask[par][2];
-        par ^= 1;
+        const unsigned long long w = sm.htask[par];
+        if (!w) break;
+        const uint32_t u = (uint32_t)(w >> 32), k = (uint32_t)(w & 0xFFFFFFFFull) >> 1;
+        const uint32_t uval = (ALG == ALG_BFS) ? ops.it : (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
         const Off b0 = a.rp[u], e0 = a.rp[u + 1];
         const Off b = b0 + (Off)k * HUB_CHUNK;
         const Off e = (e0 - b > (Off)HUB_CHUNK) ? b + HUB_CHUNK : e0;
@@ -746,6 +831,18 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, TileSmem<Off
             }
             ops.template pieces<QB>(pu, pv, pq, plo, phi, pok);
         }
+        if (threadIdx.x == 0) {
+            const unsigned long long wn = pre ? pre : hub_wait(a, c1, slot);
+            if (wn) {
+                a.hub[c1] = 0ull;
+                c1 = c2;
+                pre = c1 < a.hub_cap ? ld_relaxed64(a.hub + c1) : 0ull;
+                c2 = atomicAdd(&ctl->hub_head[slot], 1u);
+            }
+            sm.htask[par ^ 1] = wn;
+        }
+        __syncthreads();
+        par ^= 1;
     }
 }
 
@@ -850,11 +947,11 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     for (;; ++it) {
         const uint32_t slot = it % 3;
         if (n == 0 || it >= a.max_iters) break;
+        AG_PROF_MARK(it, 0);
         // decision maker, re-evaluated every sample_every iterations (inspector sampling, 26.s7-9)
         const uint8_t var = (it % a.pol.sample_every == 0 || prev_var == 0) ? select_variant(a.pol, n, 0) : prev_var;
         const uint32_t map = TUNED ? ((var >> 2) == MAP_T ? (uint32_t)MAP_T : (uint32_t)MAP_H) : (var >> 2);
         const uint32_t ws = TUNED ? (uint32_t)WS_QU : (var & 3u);
-        const uint32_t tag = a.epoch * 0x9E3779B1u + it + 1;
         if (blockIdx.x == 0 && threadIdx.x == 0) {
             if (it < a.trace_cap && a.trace_ws) {
                 a.trace_ws[it] = n;
@@ -925,7 +1022,22 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         const uint32_t ntiles = (ws == WS_BM) ? (a.V + BS - 1) / BS : (qn + tile_n - 1) / tile_n;
         const bool hubs = (map == MAP_H) && a.has_hubs;
 
-        {
+        if (AG_WARPH && TUNED && map == MAP_H && ws == WS_QU) {
+            // warp-scheduled tiles of tn <= 32 elements (>= 2 tiles per warp), claimed one ahead
+            const uint32_t nwarps = a.nblocks * WARPS_PER_CTA, lane = lane_id();
+            uint32_t tn = (qn + 2 * nwarps - 1) / (2 * nwarps);
+            tn = tn < 1u ? 1u : (tn > 32u ? 32u : tn);
+            const uint32_t nt = (qn + tn - 1) / tn;
+            uint32_t t = blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
+            while (t < nt) {
+                uint32_t nxt = 0;
+                if (lane == 0) nxt = nwarps + atomicAdd(&ctl->tile_ctr[slot], 1u);
+                const uint32_t i = t * tn + lane;
+                const bool valid = lane < tn && i < qn;
+                process_warp_tile(ops, sm, valid, valid ? qc[i] : 0u, hubs, slot);
+                t = __shfl_sync(0xffffffffu, nxt, 0);
+            }
+        } else {
             // dynamic tile scheduler: first tile static, then one atomic per tile, fetched one tile ahead
             // (double-buffered in smem; the __syncthreads_or below orders the write before the read)
             uint32_t t = blockIdx.x;
@@ -943,12 +1055,14 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
                     u = valid ? qc[i] : 0u;
                 }
                 if (__syncthreads_or(valid))  // skip empty tiles (sparse bitmap): uniform branch
-                    process_tile<TUNED>(ops, sm, map, valid, u, a.pol.cta_group, hubs, slot, tag);
+                    process_tile<TUNED>(ops, sm, map, valid, u, a.pol.cta_group, hubs, slot);
                 t = sm.tnext[par];
                 par ^= 1;
             }
         }
-        if (hubs) drain_hubs(ops, sm, slot, tag);
+        AG_PROF_MARK(it, 1);
+        if (hubs) drain_hubs(ops, sm, slot);   // (begins with __syncthreads)
+        AG_PROF_MARK(it, 2);
         ops.warp_flush(true);
         block_reduce_flush(ops, sm, ctl, slot);
         grid_barrier(ctl, a.nblocks);
