@@ -93,7 +93,13 @@ typedef struct {
     uint32_t sssp_hub_window;/* unordered SSSP: vertices with out-degree >= 64 are expanded only when within
                                 this distance of the frontier minimum (re-expanding a hub re-scans its whole
                                 list); 0 = off; AG_WINDOW_AUTO = tuned: max(1, max_weight / 50) */
-    uint32_t reserved[2];    /* must be 0 */
+    uint32_t free_ppm;       /* tuned policy, unordered: an iteration whose working set has >= free_ppm * V / 1e6
+                                elements writes its successor as a raw bitmap with fire-and-forget reductions (no
+                                claiming atomics, no queue appends; BFS without parents only) and the next
+                                iteration converts it to a queue in O(V/32) (the paper's update-vector bitmap,
+                                22.s13-14).  SSSP uses it only on graphs without the degree layout (non-skewed).
+                                0 = never; ag_policy_default: 3906 (V/256) */
+    uint32_t reserved;       /* must be 0 */
 } ag_policy;
 
 typedef struct {
@@ -231,6 +237,20 @@ ag_status ag_dist_bfs_group(ag_graph *locals, int world, uint32_t src, uint32_t 
  * (end - begin) uint32 for this rank's owned range.  Collective: all ranks call with the same src. */
 ag_status ag_dist_bfs(ag_graph local, uint32_t src, uint32_t *levels_owned, uint32_t *parents_owned,
                       const ag_policy *policy, ag_run_stats *stats, void *stream);
+/* Distributed SSSP (the algorithm is Fig. 5 unordered, PAPER.md:18.s30:
+ * every working-set node relaxes its out-edges until no distance improves).  Same destination
+ * partition; per round every rank expands the gathered global list of (vertex, distance) entries —
+ * the distance travels with the entry since only a vertex's owner holds it — over its local edges,
+ * then the improved owned vertices are exchanged: ncclAllGather of the per-rank counts (termination
+ * when all are 0) and of the (v, dist) lists padded to the largest count.  The local part must
+ * carry weights (AG_ERR_NO_WEIGHTS).  dist_owned (required) / parents_owned (nullable): (end - begin)
+ * uint32 for the owned range, host or device memory, caller-owned; AG_INF for unreached vertices.
+ * AG_ERR_OVERFLOW is reported conservatively if any relaxation exceeded 0xFFFFFFFE.  Collective. */
+ag_status ag_dist_sssp(ag_graph local, uint32_t src, uint32_t *dist_owned, uint32_t *parents_owned,
+                       const ag_policy *policy, ag_run_stats *stats, void *stream);
+/* Lock-step distributed SSSP over all ranks of a virtual group (test transport, see above). */
+ag_status ag_dist_sssp_group(ag_graph *locals, int world, uint32_t src, uint32_t **dist_owned,
+                             uint32_t **parents_owned, ag_run_stats *stats, void *stream);
 
 /* ---------------------------------------------------------------------------------------------
  * Misc

@@ -51,7 +51,8 @@ class Policy(ctypes.Structure):
                 ("workset", ctypes.c_uint32), ("kind", ctypes.c_uint32), ("t1_avg_degree", ctypes.c_uint32),
                 ("t2_ws", ctypes.c_uint64), ("t3_ppm", ctypes.c_uint32), ("sample_every", ctypes.c_uint32),
                 ("delta", ctypes.c_uint32), ("thread_tpb", ctypes.c_uint32), ("cta_group", ctypes.c_uint32),
-                ("sssp_window", ctypes.c_uint32), ("sssp_hub_window", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 2)]
+                ("sssp_window", ctypes.c_uint32), ("sssp_hub_window", ctypes.c_uint32), ("free_ppm", ctypes.c_uint32),
+                ("reserved", ctypes.c_uint32)]
 
 
 class GraphInfo(ctypes.Structure):
@@ -74,7 +75,7 @@ class RunStats(ctypes.Structure):
 EXPORTS = ["ag_policy_default", "ag_select", "ag_graph_load_csr", "ag_graph_load_csr_ex", "ag_graph_info_get",
            "ag_graph_free", "ag_bfs", "ag_sssp", "ag_graph_check", "ag_dist_unique_id", "ag_dist_init",
            "ag_dist_init_local", "ag_dist_free", "ag_dist_owned_range", "ag_dist_graph_load_csr",
-           "ag_dist_graph_load_local", "ag_dist_bfs", "ag_dist_bfs_group", "ag_set_allocator", "ag_status_string",
+           "ag_dist_graph_load_local", "ag_dist_bfs", "ag_dist_bfs_group", "ag_dist_sssp", "ag_dist_sssp_group", "ag_set_allocator", "ag_status_string",
            "ag_last_error", "ag_abi_version", "ag_kernel_launches"]
 
 _lib = None
@@ -116,6 +117,8 @@ def lib():
     L.ag_dist_init_local.argtypes = [i32, i32, vp]
     L.ag_dist_graph_load_local.argtypes = [vp, u32, u64, vp, vp, vp, ctypes.POINTER(vp)]
     L.ag_dist_bfs_group.argtypes = [vp, i32, u32, vp, vp, ctypes.POINTER(RunStats), vp]
+    L.ag_dist_sssp.argtypes = [vp, u32, vp, vp, ctypes.POINTER(Policy), ctypes.POINTER(RunStats), vp]
+    L.ag_dist_sssp_group.argtypes = [vp, i32, u32, vp, vp, ctypes.POINTER(RunStats), vp]
     L.ag_status_string.restype = ctypes.c_char_p
     L.ag_status_string.argtypes = [i32]
     L.ag_last_error.restype = ctypes.c_char_p
@@ -309,6 +312,33 @@ class DistGraph(Graph):
                                  ctypes.byref(policy) if policy is not None else None,
                                  ctypes.byref(st) if st is not None else None, ctypes.c_void_p(stream or 0)))
         return levels, parents, _stats_out(st, tr)
+
+
+    def sssp(self, src: int, dist=None, parents=None, policy=None, stats: bool = False, trace_cap: int = 0,
+             stream=None):
+        """ag_dist_sssp (collective over the NCCL communicator): returns this rank's owned slices."""
+        n = self.own[1] - self.own[0]
+        if dist is None:
+            dist = np.empty(n, np.uint32)
+        st, tr = _mkstats(stats, trace_cap)
+        _check(lib().ag_dist_sssp(self.h, int(src), _ptr(dist), _ptr(parents),
+                                  ctypes.byref(policy) if policy is not None else None,
+                                  ctypes.byref(st) if st is not None else None, ctypes.c_void_p(stream or 0)))
+        return dist, parents, _stats_out(st, tr)
+
+
+def dist_sssp_group(parts, src: int, parents: bool = False, stats: bool = False, trace_cap: int = 0):
+    """Lock-step SSSP over the ranks of a virtual group; returns (dist, parents|None, Stats) in
+    GLOBAL vertex order (owned slices concatenated)."""
+    P = len(parts)
+    dv = [np.empty(p.own[1] - p.own[0], np.uint32) for p in parts]
+    pa = [np.empty(p.own[1] - p.own[0], np.uint32) for p in parts] if parents else None
+    hs = (ctypes.c_void_p * P)(*[p.h.value for p in parts])
+    dvp = (ctypes.c_void_p * P)(*[a.ctypes.data for a in dv])
+    pap = (ctypes.c_void_p * P)(*[a.ctypes.data for a in pa]) if parents else None
+    st, tr = _mkstats(stats, trace_cap)
+    _check(lib().ag_dist_sssp_group(hs, P, int(src), dvp, pap, ctypes.byref(st) if st is not None else None, None))
+    return np.concatenate(dv), (np.concatenate(pa) if parents else None), _stats_out(st, tr)
 
 
 def dist_bfs_group(parts, src: int, parents: bool = False, stats: bool = False, trace_cap: int = 0):

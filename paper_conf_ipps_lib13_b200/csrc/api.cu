@@ -301,6 +301,12 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
     d.E = g.E;
     d.max_deg = g.info.max_deg;
     d.t2_tuned = 65536;
+    d.t_free = (p.kind == AG_POLICY_TUNED && p.free_ppm) ? ((uint64_t)g.V * p.free_ppm + 999999ull) / 1000000ull : ~0ull;
+    if (d.t_free == 0) d.t_free = 1;
+    // SSSP: free output only on non-skewed graphs (measured: ER n=2^25 21.4 -> 12.4 ms; R-MAT s22
+    // 1.59 -> 2.19 ms, the fire-and-forget red.min on power-law hot targets loses to the claiming
+    // atomicMin whose result gates the next-bitmap update)
+    d.t_free_sssp = g.info.layout == AG_LAYOUT_DEGREE ? ~0ull : d.t_free;
     return d;
 }
 
@@ -573,6 +579,7 @@ ag_status ag_policy_default(ag_policy *p, int device) {
     p->cta_group = 0;
     p->sssp_window = AG_WINDOW_AUTO;
     p->sssp_hub_window = AG_WINDOW_AUTO;
+    p->free_ppm = 3906;   // V/256 (tools/sweep.py --set free_ppm=...)
     return AG_OK;
 }
 

@@ -65,9 +65,6 @@ enum { WS_BM = 1, WS_QU = 2 };
 #ifndef AG_LONG_MIN
 #define AG_LONG_MIN 512   // hybrid mapping: lists this long go to aligned warp windows
 #endif
-#ifndef AG_WARPH
-#define AG_WARPH 0        // hybrid mapping tiles scheduled per warp (1) or per CTA (0)
-#endif
 #ifndef AG_HUBDEG
 #define AG_HUBDEG 2048
 #endif
@@ -97,6 +94,7 @@ struct alignas(128) Ctl {
     unsigned int hub_head[3];         //                 consumed hub-chunk tasks
     unsigned int stage_done[3];       //                 CTAs done producing
     unsigned long long it_edges[3];   // edges inspected in iteration (trace only)
+    unsigned int free_any[3];         // free-output iteration wrote at least one next-bitmap bit
     unsigned int pend_count;          // ordered SSSP: |pending|
     unsigned int overflow;            // a relaxation exceeded MAX_FINITE
     unsigned int iterations;
@@ -121,6 +119,8 @@ struct DevPolicy {
     uint64_t E;
     uint32_t max_deg;     // inspector: maximum out-degree (tuned policy)
     uint32_t t2_tuned;    // tuned policy: thread mapping below this |WS| on low-degree graphs
+    uint64_t t_free;      // tuned policy: free (raw-bitmap) output from this |WS| on (~0 = never), BFS
+    uint64_t t_free_sssp; //   ... SSSP (never on skewed graphs: red.min on hot targets loses, tools/gpu_free_ab.sh)
 };
 
 // The decision maker.  PAPER: Fig. 11 with readings R12/R13:
@@ -220,6 +220,9 @@ __device__ __forceinline__ uint32_t ld_ro(const uint32_t *p) { return __ldg(p); 
 __device__ __forceinline__ unsigned long long ld_ro(const unsigned long long *p) { return __ldg(p); }
 __device__ __forceinline__ void red_or(uint32_t *p, uint32_t v) {
     asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void red_min64(unsigned long long *p, unsigned long long v) {
+    asm volatile("red.relaxed.gpu.global.min.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
 __device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31u; }

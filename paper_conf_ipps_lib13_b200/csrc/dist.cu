@@ -32,7 +32,7 @@
 typedef struct ncclComm *ncclComm_t;
 typedef struct { char internal[128]; } ncclUniqueId;
 typedef enum { ncclSuccess = 0 } ncclResult_t;
-typedef enum { ncclUint8 = 1 } ncclDataType_t;
+typedef enum { ncclUint8 = 1, ncclUint32 = 3 } ncclDataType_t;
 
 namespace {
 
@@ -94,6 +94,11 @@ struct ag_dist_part {
     uint32_t *d_next = nullptr;        // next-frontier bitmap (only owned words written)
     unsigned long long *d_cnt = nullptr;
     unsigned long long *h_cnt = nullptr;  // pinned
+    // SSSP exchange buffers (allocated on the first ag_dist_sssp)
+    uint2 *d_send = nullptr;           // S entries: (owned improved vertex, its distance)
+    uint2 *d_list = nullptr;           // world * S entries: the gathered global frontier
+    unsigned *d_counts = nullptr;      // world per-rank counts (gathered)
+    unsigned *h_counts = nullptr;      // pinned copy
 };
 
 namespace ag {
@@ -105,6 +110,11 @@ void dist_graph_release(ag_graph_s *g) {
     dev_free(d->d_next, (size_t)d->gwords * 4 + 128, g->device);
     dev_free(d->d_cnt, 64, g->device);
     if (d->h_cnt) cudaFreeHost(d->h_cnt);
+    const int W = d->comm ? d->comm->world : 1;
+    dev_free(d->d_send, (size_t)d->S * 8 + 128, g->device);
+    dev_free(d->d_list, (size_t)W * d->S * 8 + 128, g->device);
+    dev_free(d->d_counts, (size_t)W * 4 + 128, g->device);
+    if (d->h_counts) cudaFreeHost(d->h_counts);
     delete d;
     g->dist = nullptr;
 }
@@ -221,6 +231,73 @@ __global__ void __launch_bounds__(BS, AG_MINB_BFS) dist_level_kernel(const TravA
     block_reduce_flush(ops, sm, ctl, slot);
 }
 
+// ---- multi-GPU SSSP on the same destination partition --------------------
+// One unordered round (Fig. 5 unordered, 18.s30: every working-set node relaxes its out-edges) on one
+// rank: the gathered global frontier is a LIST of (u, dist u) entries — the value travels with the
+// entry because only u's owner holds P[u] — expanded over the local CSR (edges u -> v with v owned)
+// with the hybrid mapping; an improved owned v gets its bit in the next bitmap (dedup) and is
+// appended to the local next queue.  Padding entries have u = INF.
+template <typename Off>
+__global__ void __launch_bounds__(BS, AG_MINB_SSSP) dist_sssp_kernel(const TravArgs<Off> a, const uint2 *list,
+                                                                     uint32_t n) {
+    __shared__ TileSmem<Off> sm;
+    Ctl *ctl = a.ctl;
+    const uint32_t slot = 0;
+    Ops<ALG_SSSP, ORD_U, Off> ops(a, 0, ~0ull, true);   // it 0: next bitmap bm[1], next queue q[1]
+    ops.wbuf = sm.wq[threadIdx.x >> 5];
+    uint32_t tile_n = (n + 2 * a.nblocks - 1) / (2 * a.nblocks);
+    tile_n = tile_n < 1u ? 1u : (tile_n > (uint32_t)BS ? (uint32_t)BS : tile_n);
+    const uint32_t ntiles = (n + tile_n - 1) / tile_n;
+    uint32_t t = blockIdx.x;
+    int par = 0;
+    while (t < ntiles) {
+        if (threadIdx.x == 0) sm.tnext[par] = a.nblocks + atomicAdd(&ctl->tile_ctr[slot], 1u);
+        const uint32_t i = t * tile_n + threadIdx.x;
+        uint2 e = make_uint2(INF, INF);
+        if (threadIdx.x < tile_n && i < n) e = list[i];
+        const bool valid = e.x != INF;
+        if (__syncthreads_or(valid))
+            process_tile<true>(ops, sm, MAP_H, valid, valid ? e.x : 0u, 32u, a.has_hubs != 0, slot, e.y, i);
+        t = sm.tnext[par];
+        par ^= 1;
+    }
+    if (a.has_hubs) drain_hubs(ops, sm, slot);
+    ops.warp_flush(true);
+    block_reduce_flush(ops, sm, ctl, slot);
+}
+
+// The rank's contribution to the next global frontier: (v, dist v) for every owned v improved in this
+// round (the local next queue, deduplicated by the bitmap), read after the round so the latest
+// distance is sent; clears the next-bitmap words for the following round.
+__global__ void dist_sssp_collect_kernel(const uint32_t *q, const unsigned *qlen, const unsigned long long *P,
+                                         uint32_t *next_bm, uint2 *send, unsigned *count) {
+    const uint32_t n = *qlen;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+        const uint32_t v = q[i];
+        send[i] = make_uint2(v, (uint32_t)(P[v] >> 32));
+        next_bm[v >> 5] = 0u;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) *count = n;
+}
+
+__global__ void dist_sssp_init_kernel(unsigned long long *P, uint32_t *next_bm, uint32_t V, uint32_t gwords,
+                                      uint32_t src, uint32_t own_b, uint32_t own_e) {
+    const uint32_t gt = blockIdx.x * blockDim.x + threadIdx.x, gs = gridDim.x * blockDim.x;
+    for (uint32_t v = gt; v < V; v += gs)
+        P[v] = (v == src && src >= own_b && src < own_e) ? (unsigned long long)src : INF64;   // dist 0, parent src
+    for (uint32_t wi = gt; wi < gwords; wi += gs) next_bm[wi] = 0u;
+}
+
+// owned slice -> caller arrays: dist, parent (INF for unreached)
+__global__ void dist_sssp_out_kernel(const unsigned long long *P, uint32_t b, uint32_t e, uint32_t *dist,
+                                     uint32_t *parent) {
+    for (uint32_t v = b + blockIdx.x * blockDim.x + threadIdx.x; v < e; v += gridDim.x * blockDim.x) {
+        const unsigned long long pv = P[v];
+        dist[v - b] = (uint32_t)(pv >> 32);
+        if (parent) parent[v - b] = pv == INF64 ? INF : (uint32_t)pv;
+    }
+}
+
 // ------------------------------------------------------------------------------------------------
 // host side
 // ------------------------------------------------------------------------------------------------
@@ -299,6 +376,60 @@ ag_status launch_level(ag_graph_s *g, uint32_t L, uint32_t *parent_local, cudaSt
     cudaError_t e = cudaLaunchCooperativeKernel((const void *)fn, dim3(a.nblocks), dim3(BS), args, 0, st);
     note_launch(1);
     return cuda_status(e, "dist level");
+}
+
+// SSSP scratch: packed state P (V), exchange buffers
+ag_status dist_sssp_scratch(ag_graph_s *g) {
+    ag_status s;
+    ag_dist_part *d = g->dist;
+    const int W = d->comm->world;
+    if (!g->d_P && (s = dev_alloc((void **)&g->d_P, (size_t)g->V * 8 + 128, g->device)) != AG_OK) return s;
+    if (!d->d_send && (s = dev_alloc((void **)&d->d_send, (size_t)d->S * 8 + 128, g->device)) != AG_OK) return s;
+    if (!d->d_list && (s = dev_alloc((void **)&d->d_list, (size_t)W * d->S * 8 + 128, g->device)) != AG_OK) return s;
+    if (!d->d_counts && (s = dev_alloc((void **)&d->d_counts, (size_t)W * 4 + 128, g->device)) != AG_OK) return s;
+    if (!d->h_counts && cudaMallocHost(&d->h_counts, (size_t)W * 4 + 64) != cudaSuccess)
+        return set_error(AG_ERR_OOM, "pinned alloc");
+    return AG_OK;
+}
+
+template <typename Off>
+ag_status launch_sssp_round(ag_graph_s *g, const uint2 *list, uint32_t n, cudaStream_t st) {
+    ag_dist_part *d = g->dist;
+    TravArgs<Off> a;
+    memset(&a, 0, sizeof a);
+    a.rp = (const Off *)g->d_rp;
+    a.cw = g->d_cw;
+    a.V = g->V;
+    a.nwords = d->gwords;
+    a.P = g->d_P;
+    a.bm[0] = a.bm[1] = a.bm[2] = d->d_next;
+    a.q[0] = a.q[2] = g->d_q[0];
+    a.q[1] = g->d_q[1];
+    a.hub = g->d_hub;
+    a.hub_cap = g->hub_cap;
+    a.ctl = (Ctl *)g->d_ctl;
+    a.epoch = ++g->epoch;
+    a.has_hubs = g->info.max_deg >= HUB_DEG;
+    a.ulist = list;
+    auto fn = dist_sssp_kernel<Off>;
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, BS, 0);
+    if (occ < 1) return set_error(AG_ERR_CUDA, "dist sssp kernel does not fit");
+    a.nblocks = (uint32_t)(occ * g->num_sms);
+    cudaMemsetAsync((char *)g->d_ctl + offsetof(Ctl, q_len), 0, offsetof(Ctl, it_edges) - offsetof(Ctl, q_len), st);
+    void *args[] = {(void *)&a, (void *)&list, (void *)&n};
+    cudaError_t e = cudaLaunchCooperativeKernel((const void *)fn, dim3(a.nblocks), dim3(BS), args, 0, st);
+    note_launch(1);
+    if (e != cudaSuccess) return cuda_status(e, "dist sssp round");
+    dist_sssp_collect_kernel<<<g->num_sms * 2, 256, 0, st>>>(g->d_q[1], &((Ctl *)g->d_ctl)->q_len[1], g->d_P, d->d_next,
+                                                             d->d_send, d->d_counts + d->comm->rank);
+    note_launch(1);
+    return cuda_status(cudaGetLastError(), "dist sssp collect");
+}
+
+ag_status run_sssp_round(ag_graph_s *g, const uint2 *list, uint32_t n, cudaStream_t st) {
+    return g->offs32 ? launch_sssp_round<uint32_t>(g, list, n, st)
+                     : launch_sssp_round<unsigned long long>(g, list, n, st);
 }
 
 ag_status run_level(ag_graph_s *g, uint32_t L, uint32_t *parent_local, cudaStream_t st) {
@@ -585,6 +716,131 @@ ag_status dist_bfs_driver(std::vector<ag_graph_s *> &parts, uint32_t src, uint32
     return AG_OK;
 }
 
+// Lock-step unordered SSSP over the participating ranks of THIS process.  Per round: every rank
+// expands the same gathered list, collects its improved owned vertices, the per-rank counts are
+// all-gathered (termination: all zero), then the (v, dist) lists padded to the largest count.
+ag_status dist_sssp_driver(std::vector<ag_graph_s *> &parts, uint32_t src, uint32_t **dist_owned,
+                           uint32_t **parents_owned, ag_run_stats *stats, cudaStream_t st) {
+    const int P = (int)parts.size();
+    ag_status s;
+    for (auto *g : parts) {
+        cudaSetDevice(g->device);
+        if (!g->d_cw) return set_error(AG_ERR_NO_WEIGHTS, "SSSP on an unweighted distributed graph");
+        if ((s = dist_scratch(g)) != AG_OK) return s;
+        if ((s = dist_sssp_scratch(g)) != AG_OK) return s;
+    }
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    if (stats) {
+        cudaEventCreate(&e0);
+        cudaEventCreate(&e1);
+        cudaEventRecord(e0, st);
+    }
+    const uint32_t V = parts[0]->V;
+    const int world = parts[0]->dist->comm->world;
+    const bool nccl = P == 1 && parts[0]->dist->comm->nccl;
+    const uint2 first = make_uint2(src, 0u);
+    for (auto *g : parts) {
+        ag_dist_part *d = g->dist;
+        dist_sssp_init_kernel<<<g->num_sms * 4, 256, 0, st>>>(g->d_P, d->d_next, V, d->gwords, src, d->own_b, d->own_e);
+        cudaMemsetAsync(g->d_ctl, 0, offsetof(Ctl, q_len), st);
+        cudaMemsetAsync((char *)g->d_ctl + offsetof(Ctl, vexp), 0, 16, st);
+        cudaMemsetAsync((char *)g->d_ctl + offsetof(Ctl, overflow), 0, 4, st);
+        cudaMemcpyAsync(d->d_list, &first, sizeof first, cudaMemcpyHostToDevice, st);
+        note_launch(1);
+    }
+    uint32_t n = 1, R = 0;   // entries of the gathered list (with padding), rounds
+    uint64_t front = 1;      // real entries
+    const uint32_t tcap = stats ? stats->trace_cap : 0;
+    for (;; ++R) {
+        if (stats && R < tcap && stats->trace_ws) stats->trace_ws[R] = (uint32_t)front;
+        for (auto *g : parts)
+            if ((s = run_sssp_round(g, g->dist->d_list, n, st)) != AG_OK) return s;
+        // counts: every rank's count to every rank
+        if (nccl) {
+            ag_dist_part *d = parts[0]->dist;
+            ncclResult_t r = g_nccl.AllGather(d->d_counts + d->comm->rank, d->d_counts, 1, ncclUint32, d->comm->nccl, st);
+            if ((s = nccl_status(r, "ncclAllGather(counts)")) != AG_OK) return s;
+        } else {
+            for (auto *gd : parts)
+                for (auto *gs : parts)
+                    if (gd != gs)
+                        cudaMemcpyAsync(gd->dist->d_counts + gs->dist->comm->rank, gs->dist->d_counts + gs->dist->comm->rank, 4,
+                                        cudaMemcpyDeviceToDevice, st);
+        }
+        ag_dist_part *d0 = parts[0]->dist;
+        cudaMemcpyAsync(d0->h_counts, d0->d_counts, (size_t)world * 4, cudaMemcpyDeviceToHost, st);
+        cudaError_t ce = cudaStreamSynchronize(st);
+        if (ce != cudaSuccess) return cuda_status(ce, "dist sssp round");
+        uint32_t maxc = 0;
+        front = 0;
+        for (int r = 0; r < world; ++r) {
+            maxc = d0->h_counts[r] > maxc ? d0->h_counts[r] : maxc;
+            front += d0->h_counts[r];
+        }
+        if (front == 0 || R > 4u * V + 64u) break;
+        // pad every send list to maxc with (INF, INF), then gather rank-ordered into the global list
+        for (auto *g : parts) {
+            ag_dist_part *d = g->dist;
+            const uint32_t c = d0->h_counts[d->comm->rank];
+            if (c < maxc) cudaMemsetAsync(d->d_send + c, 0xFF, (size_t)(maxc - c) * 8, st);
+        }
+        if (nccl) {
+            ag_dist_part *d = parts[0]->dist;
+            ncclResult_t r = g_nccl.AllGather(d->d_send, d->d_list, (size_t)maxc * 8, ncclUint8, d->comm->nccl, st);
+            if ((s = nccl_status(r, "ncclAllGather(frontier)")) != AG_OK) return s;
+        } else {
+            for (auto *gd : parts)
+                for (auto *gs : parts)
+                    cudaMemcpyAsync(gd->dist->d_list + (size_t)gs->dist->comm->rank * maxc, gs->dist->d_send,
+                                    (size_t)maxc * 8, cudaMemcpyDeviceToDevice, st);
+        }
+        n = (uint32_t)world * maxc;
+    }
+    for (int r = 0; r < P; ++r) {
+        ag_graph_s *g = parts[r];
+        ag_dist_part *d = g->dist;
+        if (d->own_e > d->own_b && dist_owned && dist_owned[r]) {
+            // device outputs directly; host outputs through the queue buffer q[0] as staging
+            uint32_t *dd = dist_owned[r], *pp = parents_owned ? parents_owned[r] : nullptr;
+            const bool dh = !is_device_ptr(dd), ph = pp && !is_device_ptr(pp);
+            const size_t cnt = d->own_e - d->own_b;
+            uint32_t *sd = dh ? g->d_q[0] : dd, *sp = ph ? g->d_q[1] : pp;   // staging: V entries each
+            dist_sssp_out_kernel<<<g->num_sms * 2, 256, 0, st>>>(g->d_P, d->own_b, d->own_e, sd, sp);
+            note_launch(1);
+            if (dh) cudaMemcpyAsync(dd, sd, cnt * 4, cudaMemcpyDeviceToHost, st);
+            if (ph) cudaMemcpyAsync(pp, sp, cnt * 4, cudaMemcpyDeviceToHost, st);
+        }
+    }
+    if (stats) cudaEventRecord(e1, st);
+    cudaError_t ce = cudaStreamSynchronize(st);
+    if (ce != cudaSuccess) return cuda_status(ce, "dist sssp");
+    unsigned long long vx = 0, ex = 0;
+    bool ovf = false;
+    for (auto *g : parts) {
+        Ctl c;
+        cudaMemcpy(&c, g->d_ctl, sizeof c, cudaMemcpyDeviceToHost);
+        vx += c.vexp;
+        ex += c.eexp;
+        ovf |= c.overflow != 0;
+        if (c.aborted) return set_error(AG_ERR_CUDA, "dist sssp aborted (code %u)", c.aborted);
+    }
+    if (stats) {
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        cudaEventDestroy(e0);
+        cudaEventDestroy(e1);
+        stats->iterations = R + 1;
+        stats->device_ms = ms;
+        stats->vertices_expanded = vx;
+        stats->edges_inspected = ex;
+        stats->trace_len = (R + 1) < tcap ? (R + 1) : tcap;
+    }
+    // a relaxation past 0xFFFFFFFE was dropped somewhere: reported conservatively (the distributed path
+    // has no exact re-check like the single-GPU one; the outputs are still written)
+    if (ovf) return set_error(AG_ERR_OVERFLOW, "a distance exceeds 0xFFFFFFFE");
+    return AG_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -616,6 +872,36 @@ ag_status ag_dist_bfs_group(ag_graph *locals, int world, uint32_t src, uint32_t 
     if (stats && stats->struct_size != sizeof(ag_run_stats)) return set_error(AG_ERR_INVALID_ARG, "stats size");
     cudaSetDevice(parts[0]->device);
     return dist_bfs_driver(parts, src, levels_owned, parents_owned, stats, (cudaStream_t)stream);
+}
+
+ag_status ag_dist_sssp(ag_graph local, uint32_t src, uint32_t *dist_owned, uint32_t *parents_owned,
+                       const ag_policy *policy, ag_run_stats *stats, void *stream) {
+    (void)policy;
+    if (!local || !local->dist) return set_error(AG_ERR_INVALID_ARG, "not a distributed graph");
+    if (!dist_owned) return set_error(AG_ERR_INVALID_ARG, "dist_owned is NULL");
+    if (src >= local->V) return set_error(AG_ERR_SRC_RANGE, "src %u >= V %u", src, local->V);
+    if (stats && stats->struct_size != sizeof(ag_run_stats)) return set_error(AG_ERR_INVALID_ARG, "stats size");
+    if (local->dist->comm->group) return set_error(AG_ERR_INVALID_ARG, "virtual-group graph: use ag_dist_sssp_group");
+    std::vector<ag_graph_s *> parts{local};
+    uint32_t *dv[1] = {dist_owned};
+    uint32_t *pa[1] = {parents_owned};
+    cudaSetDevice(local->device);
+    return dist_sssp_driver(parts, src, dv, parents_owned ? pa : nullptr, stats, (cudaStream_t)stream);
+}
+
+ag_status ag_dist_sssp_group(ag_graph *locals, int world, uint32_t src, uint32_t **dist_owned,
+                             uint32_t **parents_owned, ag_run_stats *stats, void *stream) {
+    if (!locals || world < 1 || !dist_owned) return set_error(AG_ERR_INVALID_ARG, "bad args");
+    std::vector<ag_graph_s *> parts;
+    for (int r = 0; r < world; ++r) {
+        if (!locals[r] || !locals[r]->dist || !locals[r]->dist->comm->group || locals[r]->dist->comm->rank != r)
+            return set_error(AG_ERR_INVALID_ARG, "locals[%d] is not rank %d of a virtual group", r, r);
+        parts.push_back(locals[r]);
+    }
+    if (src >= parts[0]->V) return set_error(AG_ERR_SRC_RANGE, "src out of range");
+    if (stats && stats->struct_size != sizeof(ag_run_stats)) return set_error(AG_ERR_INVALID_ARG, "stats size");
+    cudaSetDevice(parts[0]->device);
+    return dist_sssp_driver(parts, src, dist_owned, parents_owned, stats, (cudaStream_t)stream);
 }
 
 }  // extern "C"

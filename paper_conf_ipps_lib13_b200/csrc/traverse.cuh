@@ -75,6 +75,8 @@ struct TravArgs {
     uint32_t epoch;
     uint32_t max_iters;
     uint32_t has_hubs;
+    const uint2 *ulist;         // listed working set (multi-GPU SSSP): entry i = (u, dist of u); the value
+                                // travels with the entry, hub tasks carry the entry index (nullptr: off)
 };
 
 // per-warp staging capacity: one batch appends at most 32 x (edges per thread per batch), plus < 32 left over
@@ -94,7 +96,7 @@ struct __align__(16) TileSmem {
     unsigned long long red64[2][WARPS_PER_CTA];
     uint32_t red32[2][WARPS_PER_CTA];
     int redi[WARPS_PER_CTA];
-    uint32_t wsc[WARPS_PER_CTA][32];   // warp-tile piece scan (warp-scheduled hybrid mapping)
+    uint32_t redany[WARPS_PER_CTA];
     uint32_t tnext[2];
     uint32_t bcast;
     unsigned long long htask[2];   // hub-drain task slots (task word, 0 = drained)
@@ -124,6 +126,8 @@ struct Ops {
     uint32_t vmin;
     int dpend;
     bool ovf;
+    bool freeo = false;     // free output: next working set = raw bitmap by fire-and-forget reductions
+    bool any = false;       //   ... and this thread set at least one bit of it
 
     __device__ Ops(const TravArgs<Off> &a_, uint32_t it_, uint64_t hi_, bool append_)
         : a(a_), it(it_), hi(hi_), append_next(append_), fenced(ALG == ALG_SSSP && ORD == ORD_O && a_.pol.delta > 1),
@@ -140,6 +144,8 @@ struct Ops {
         bool ex = true;
         if constexpr (ALG == ALG_BFS) {
             uval = it;  // the frontier of iteration it is exactly level it (level-synchronous, 26.s33)
+        } else if (a.ulist) {
+            // listed entry: uval (the sender's distance of u) was set by the caller; every entry expands
         } else {
             uint32_t t = (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
             uval = t;
@@ -170,8 +176,13 @@ struct Ops {
                 ex = false;
                 vmin = min(vmin, t);
                 const uint32_t m = 1u << (u & 31);
-                const bool fresh = !(atomicOr(bm_next + (u >> 5), m) & m);
-                warp_append(q_next, qlen_next, fresh, u);
+                if (freeo) {
+                    red_or(bm_next + (u >> 5), m);
+                    any = true;
+                } else {
+                    const bool fresh = !(atomicOr(bm_next + (u >> 5), m) & m);
+                    warp_append(q_next, qlen_next, fresh, u);
+                }
             }
         }
         if (ex) {
@@ -184,6 +195,18 @@ struct Ops {
             deg = 0;
         }
         return ex;
+    }
+
+    // The (u, uval) of a hub task key: the vertex itself, or the listed entry index
+    __device__ __forceinline__ void task_vertex(uint32_t key, uint32_t &u, uint32_t &uval) const {
+        if (a.ulist) {
+            const uint2 e = a.ulist[key];
+            u = e.x;
+            uval = e.y;
+        } else {
+            u = key;
+            uval = (ALG == ALG_BFS) ? it : (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
+        }
     }
 
     // Status word of v, read before deciding to update.  Plain (L1-cacheable) load: a stale value is
@@ -271,6 +294,23 @@ struct Ops {
             }
         }
         if (CONV && !__any_sync(0xffffffffu, cm != 0)) return 0u;
+        if (freeo) {
+            // free output: every candidate marks v in the next bitmap with a reduction that returns
+            // nothing (the update vector, 22.s13-14); BFS levels are assigned when the next iteration
+            // compacts the bitmap, SSSP lowers the packed (dist, parent) word with red.min
+#pragma unroll
+            for (int j = 0; j < NB; ++j) {
+                if ((cm >> j) & 1u) {
+                    if constexpr (ALG == ALG_SSSP) {
+                        red_min64(&a.P[v[j]], (nd[j] << 32) | u[j]);            // m.distance = d (l.8)
+                        vmin = min(vmin, (uint32_t)nd[j]);
+                    }
+                    red_or(bm_next + (v[j] >> 5), 1u << (v[j] & 31));           // ws.add(m)       (l.9)
+                }
+            }
+            any |= cm != 0;
+            return 0u;
+        }
         uint32_t nwm = 0;
         if constexpr (ALG == ALG_BFS) {
             // (2) every claiming atomic of the batch issued back to back, (3) results resolved
@@ -341,7 +381,6 @@ struct Ops {
     __device__ __forceinline__ void batch(const uint32_t (&u)[NB], const uint32_t (&uv)[NB], const Off (&e)[NB],
                                           const bool (&ok)[NB]) {
         uint32_t v[NB], wt[NB];
-        St st[NB];
 #pragma unroll
         for (int j = 0; j < NB; ++j) {
             if constexpr (ALG == ALG_SSSP) {
@@ -353,15 +392,6 @@ struct Ops {
                 wt[j] = 1u;
             }
         }
-#if defined(AG_EXPERIMENT) && AG_EXPERIMENT == 1   // ceiling experiment: stream only
-        {
-            uint32_t acc = 0;
-#pragma unroll
-            for (int j = 0; j < NB; ++j) acc += v[j] + wt[j];
-            if (acc == 0xFFFFFFFFu) ovf = true;
-            return;
-        }
-#endif
         batch_vals<NB, STAGED>(u, uv, v, wt, ok);
     }
 
@@ -372,15 +402,6 @@ struct Ops {
         St st[NB];
 #pragma unroll
         for (int j = 0; j < NB; ++j) st[j] = ok[j] ? status(v[j]) : (St)0;
-#if defined(AG_EXPERIMENT) && AG_EXPERIMENT == 2   // ceiling experiment: stream + status, no update
-        {
-            uint32_t acc = 0;
-#pragma unroll
-            for (int j = 0; j < NB; ++j) acc += (uint32_t)st[j];
-            if (acc == 0x12345u) ovf = true;
-            return;
-        }
-#endif
         if constexpr (STAGED) {
             const uint32_t nwm = update_batch<NB, true>(u, uv, v, wt, st, ok);  // bit j: v[j] entered the next WS
             if (__any_sync(0xffffffffu, nwm != 0)) {   // rare on the big levels: skip the ballots otherwise
@@ -434,13 +455,25 @@ struct Ops {
                 vv[j * QE + k] = pv[j];
             }
         }
-#if defined(AG_EXPERIMENT) && AG_EXPERIMENT == 1   // ceiling experiment: stream only
+#if defined(AG_EXPERIMENT) && (AG_EXPERIMENT == 11 || AG_EXPERIMENT == 12)
+        // marginal-cost experiments (same frontiers, extra work): 11 repeats the 128-bit CSR loads,
+        // 12 repeats the CSR loads and the status gathers
         {
             uint32_t acc = 0;
 #pragma unroll
-            for (int j = 0; j < N; ++j) acc += ok[j] ? v[j] : 0u;
-            if (acc == 0xFFFFFFFFu) ovf = true;
-            return;
+            for (int j = 0; j < NQ; ++j) {
+                uint4 c = pok[j] ? ld_stream4(reinterpret_cast<const uint4 *>(
+                                                  (ALG == ALG_SSSP) ? (const void *)(a.cw + pq[j] * QE + 0)
+                                                                    : (const void *)(a.col + pq[j] * QE + 0)),
+                                              pol_keep)
+                                 : make_uint4(0u, 0u, 0u, 0u);
+                if (AG_EXPERIMENT == 12) {
+                    if (pok[j]) acc += status(c.x) + status(c.z) + ((ALG == ALG_SSSP) ? 0u : status(c.y) + status(c.w));
+                } else {
+                    acc += c.x ^ c.y ^ c.z ^ c.w;
+                }
+            }
+            if (acc == 0x9E3779B1u) ovf = true;
         }
 #endif
         batch_vals<N, true>(uu, vv, v, wt, ok);
@@ -540,7 +573,9 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, Tile
     uint32_t vmin = warp_min(ops.vmin);
     int dp = warp_sum(ops.dpend);
     unsigned ovf = __any_sync(0xffffffffu, ops.ovf);
+    unsigned anyw = __any_sync(0xffffffffu, ops.any);
     if (lane == 0) {
+        sm.redany[wid] = anyw;
         sm.red64[0][wid] = ne;
         sm.red64[1][wid] = nv;
         sm.red32[0][wid] = vmin;
@@ -550,9 +585,10 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, Tile
     __syncthreads();
     if (threadIdx.x == 0) {
         unsigned long long se = 0, sv = 0;
-        uint32_t mn = INF, ov = 0;
+        uint32_t mn = INF, ov = 0, an = 0;
         int sd = 0;
         for (int i = 0; i < WARPS_PER_CTA; ++i) {
+            an |= sm.redany[i];
             se += sm.red64[0][i];
             sv += sm.red64[1][i];
             mn = min(mn, sm.red32[0][i]);
@@ -569,6 +605,7 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, Tile
             if (ORD == ORD_O && sd) atomicAdd(&ctl->pend_count, (unsigned)sd);
         }
         if (ov) ctl->overflow = 1;
+        if (an) ctl->free_any[(slot + 1) % 3] = 1u;
     }
     // (the following grid barrier begins with __syncthreads)
 }
@@ -578,10 +615,12 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, Tile
 // ------------------------------------------------------------------------------------------------
 template <bool TUNED, int ALG, int ORD, typename Off>
 __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<Off> &sm, uint32_t map,
-                                             bool valid, uint32_t u, uint32_t group, bool hubs, uint32_t slot) {
+                                             bool valid, uint32_t u, uint32_t group, bool hubs, uint32_t slot,
+                                             uint32_t uval_in = 0, uint32_t key = 0xFFFFFFFFu) {
     const TravArgs<Off> &a = ops.a;
     Off beg = 0;
-    uint32_t deg = 0, uval = 0;
+    uint32_t deg = 0, uval = uval_in;
+    if (key == 0xFFFFFFFFu) key = u;   // hub-task key: the vertex, or its listed entry index
     bool ex = valid && ops.gate(u, beg, deg, uval);
     if (!ex) deg = 0;
     const uint32_t tid = threadIdx.x, lane = lane_id();
@@ -632,7 +671,7 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<O
         // slot after reading it, so a nonzero word is always a task of the current iteration
         for (uint32_t k = 0; k < nch; ++k) {
             uint32_t idx = base + k;
-            if (idx < a.hub_cap) st_relaxed64(a.hub + idx, ((unsigned long long)u << 32) | ((unsigned long long)k << 1) | 1ull);
+            if (idx < a.hub_cap) st_relaxed64(a.hub + idx, ((unsigned long long)key << 32) | ((unsigned long long)k << 1) | 1ull);
             else a.ctl->aborted = 2;
         }
     }
@@ -683,79 +722,22 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<O
             plo[j] = bo;
             phi[j] = bo + sm.deg[lo];
             pq[j] = bo / QE + (p - sm.scan[lo]);   // aligned piece index
+#if defined(AG_EXPERIMENT) && AG_EXPERIMENT == 13   // marginal cost of the owner search: search twice
+            {
+                uint32_t lo2 = 0, hi2 = BS;
+                const uint32_t p2 = p ^ (uint32_t)(pq[j] & 1);
+#pragma unroll
+                for (int step = 0; step < LOG_BS; ++step) {
+                    const uint32_t mid = (lo2 + hi2) >> 1;
+                    if (sm.scan[mid] <= p2) lo2 = mid; else hi2 = mid;
+                }
+                if (lo2 == 0xFFFFu) ops.ovf = true;
+            }
+#endif
         }
         ops.template pieces<QB>(pu, pv, pq, plo, phi, pok);
     }
     // no trailing barrier: the next tile's __syncthreads_or orders the reuse of the tile arrays
-}
-
-// Warp-scheduled hybrid mapping (AG_WARPH): the same load-balanced gather over aligned 16-byte
-// pieces as process_tile, but each warp claims its own tiles of <= 32 working-set elements (one
-// atomic per warp tile), scans its lanes' piece counts with shuffles and finds piece owners with a
-// 5-step search over its own 32 scan entries: no CTA barrier in the expansion, so a warp stalled on
-// gathers never holds up the other warps of its CTA.  Hub lists still go to the CTA-level drain.
-template <int ALG, int ORD, typename Off>
-__device__ __forceinline__ void process_warp_tile(Ops<ALG, ORD, Off> &ops, TileSmem<Off> &sm, bool valid, uint32_t u,
-                                                  bool hubs, uint32_t slot) {
-    const TravArgs<Off> &a = ops.a;
-    Off beg = 0;
-    uint32_t deg = 0, uval = 0;
-    const bool ex = valid && ops.gate(u, beg, deg, uval);
-    if (!ex) deg = 0;
-    const uint32_t tid = threadIdx.x, lane = lane_id(), wid = tid >> 5;
-    const bool is_hub = hubs && deg >= HUB_DEG;
-    if (is_hub) {
-        const uint32_t nch = (deg + HUB_CHUNK - 1) / HUB_CHUNK;
-        uint32_t base = atomicAdd(&a.ctl->hub_tail[slot], nch);
-        for (uint32_t k = 0; k < nch; ++k) {
-            uint32_t idx = base + k;
-            if (idx < a.hub_cap) st_relaxed64(a.hub + idx, ((unsigned long long)u << 32) | ((unsigned long long)k << 1) | 1ull);
-            else a.ctl->aborted = 2;
-        }
-    }
-    constexpr uint32_t QE = Ops<ALG, ORD, Off>::QE;
-    constexpr int QB = Ops<ALG, ORD, Off>::QB;
-    const uint32_t d = is_hub ? 0u : deg;
-    const uint32_t np = d ? (uint32_t)((beg + d + QE - 1) / QE - beg / QE) : 0u;
-    uint32_t x = np;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        uint32_t xo = __shfl_up_sync(0xffffffffu, x, o);
-        if (lane >= (unsigned)o) x += xo;
-    }
-    const uint32_t NP = __shfl_sync(0xffffffffu, x, 31);
-    if (NP == 0) return;
-    __syncwarp();   // the previous warp tile's readers are done with the per-warp arrays
-    sm.u[tid] = u;
-    sm.uval[tid] = uval;
-    sm.beg[tid] = beg;
-    sm.deg[tid] = d;
-    uint32_t *sc = sm.wsc[wid];
-    sc[lane] = x - np;
-    __syncwarp();
-    const uint32_t w0 = wid * 32;
-    for (uint32_t base = 0; base < NP; base += QB * 32) {
-        uint32_t pu[QB], pv[QB];
-        Off pq[QB], plo[QB], phi[QB];
-        bool pok[QB];
-#pragma unroll
-        for (int j = 0; j < QB; ++j) {
-            const uint32_t p = base + j * 32 + lane;
-            pok[j] = p < NP;
-            uint32_t lo = 0;   // owner: the largest lane i with scan[i] <= p
-#pragma unroll
-            for (int step = 16; step > 0; step >>= 1)
-                if (sc[lo + step] <= p) lo += step;
-            const uint32_t o = w0 + lo;
-            pu[j] = sm.u[o];
-            pv[j] = sm.uval[o];
-            const Off bo = sm.beg[o];
-            plo[j] = bo;
-            phi[j] = bo + sm.deg[o];
-            pq[j] = bo / QE + (p - sc[lo]);   // aligned piece index
-        }
-        ops.template pieces<QB>(pu, pv, pq, plo, phi, pok);
-    }
 }
 
 // Wait for hub task t of this iteration: its word, or 0 once the producers are all done and t is
@@ -808,8 +790,9 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, TileSmem<Off
     for (;;) {
         const unsigned long long w = sm.htask[par];
         if (!w) break;
-        const uint32_t u = (uint32_t)(w >> 32), k = (uint32_t)(w & 0xFFFFFFFFull) >> 1;
-        const uint32_t uval = (ALG == ALG_BFS) ? ops.it : (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
+        const uint32_t k = (uint32_t)(w & 0xFFFFFFFFull) >> 1;
+        uint32_t u, uval;
+        ops.task_vertex((uint32_t)(w >> 32), u, uval);
         const Off b0 = a.rp[u], e0 = a.rp[u + 1];
         const Off b = b0 + (Off)k * HUB_CHUNK;
         const Off e = (e0 - b > (Off)HUB_CHUNK) ? b + HUB_CHUNK : e0;
@@ -843,6 +826,57 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, TileSmem<Off
         }
         __syncthreads();
         par ^= 1;
+    }
+}
+
+// Free-output successor -> queue: O(V/32) compaction of the raw next bitmap (the "converted in
+// O(V/32)" working-set switch; prefix scan instead of per-element atomics, 22.s24).  Each thread
+// takes one word per step, one atomic per CTA step.  BFS keeps only the unvisited bits, marks them
+// visited and assigns their level (the bitmap held candidates, not claims); SSSP keeps every bit.
+// Every word is cleared for reuse.
+template <int ALG, typename Off>
+__device__ __forceinline__ void compact_raw(const TravArgs<Off> &a, TileSmem<Off> &sm, uint32_t *bm, uint32_t lvl,
+                                            uint32_t *q, unsigned *qlen) {
+    const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
+    for (uint32_t w0 = blockIdx.x * BS; w0 < a.nwords; w0 += a.nblocks * BS) {
+        const uint32_t wi = w0 + threadIdx.x;
+        uint32_t word = wi < a.nwords ? bm[wi] : 0u;
+        if (word) {
+            bm[wi] = 0u;
+            if constexpr (ALG == ALG_BFS) {
+                const uint32_t vw = a.vis[wi];
+                word &= ~vw;
+                if (word) a.vis[wi] = vw | word;
+            }
+        }
+        const uint32_t c = __popc(word);
+        uint32_t x = c;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= (unsigned)o) x += y;
+        }
+        if (lane == 31) sm.red32[0][wid] = x;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            uint32_t tot = 0;
+            for (int i = 0; i < WARPS_PER_CTA; ++i) {
+                const uint32_t t = sm.red32[0][i];
+                sm.red32[1][i] = tot;
+                tot += t;
+            }
+            sm.bcast = tot ? atomicAdd(qlen, tot) : 0u;
+        }
+        __syncthreads();
+        uint32_t pos = sm.bcast + sm.red32[1][wid] + x - c;
+        while (word) {
+            const int b = __ffs(word) - 1;
+            word &= word - 1;
+            const uint32_t v = wi * 32 + b;
+            q[pos++] = v;
+            if constexpr (ALG == ALG_BFS) a.level[v] = lvl;   // m.level = level (Fig. 4 l.9)
+        }
+        __syncthreads();   // red32 / bcast reuse
     }
 }
 
@@ -901,16 +935,6 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             a.P[v] = (v == src) ? (unsigned long long)src : INF64;   // dist 0, parent src
     }
     const uint32_t sbit = 1u << (src & 31), sword = src >> 5;
-#ifdef AG_EXPERIMENT   // ceiling experiments: one full sweep over every vertex (all already visited)
-    for (uint32_t wi = gtid; wi < a.nwords; wi += gthreads) {
-        const uint32_t full = (wi * 32 + 32 <= a.V) ? 0xFFFFFFFFu : ((1u << (a.V & 31)) - 1u);
-        a.bm[0][wi] = full;
-        a.bm[1][wi] = 0u;
-        a.bm[2][wi] = 0u;
-        if (ALG == ALG_BFS) a.vis[wi] = full;
-    }
-    if (false)
-#endif
     for (uint32_t wi = gtid; wi < a.nwords; wi += gthreads) {
         a.bm[0][wi] = (wi == sword) ? sbit : 0u;
         if (ROT) {
@@ -929,6 +953,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             ctl->hub_head[s] = 0;
             ctl->stage_done[s] = 0;
             ctl->it_edges[s] = 0;
+            ctl->free_any[s] = 0;
         }
         ctl->pend_count = 1;
         ctl->overflow = 0;
@@ -944,8 +969,14 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     uint8_t prev_var = 0;
     uint32_t n_prev = 0;
     uint32_t it = 0;
+    bool in_raw = false;   // this iteration's working set is the raw bitmap of a free-output iteration
     for (;; ++it) {
         const uint32_t slot = it % 3;
+        if (TUNED && in_raw) {
+            compact_raw<ALG>(a, sm, a.bm[slot], it, a.q[slot], &ctl->q_len[slot]);
+            grid_barrier(ctl, a.nblocks);
+            n = ld_relaxed(&ctl->q_len[slot]);
+        }
         if (n == 0 || it >= a.max_iters) break;
         AG_PROF_MARK(it, 0);
         // decision maker, re-evaluated every sample_every iterations (inspector sampling, 26.s7-9)
@@ -967,6 +998,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             ctl->hub_head[rs] = 0;
             ctl->stage_done[rs] = 0;
             ctl->it_edges[rs] = 0;
+            ctl->free_any[rs] = 0;
         }
 
         uint64_t hi = ~0ull;
@@ -1005,6 +1037,9 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
 
         Ops<ALG, ORD, Off> ops(a, it, hi, append);
         ops.wbuf = sm.wq[threadIdx.x >> 5];
+        // free output (tuned, unordered, big working sets; BFS only without parents: a claim decides them)
+        ops.freeo = TUNED && ROT && (ALG == ALG_SSSP ? (uint64_t)qn >= a.pol.t_free_sssp
+                                                     : ((uint64_t)qn >= a.pol.t_free && a.parent == nullptr));
         if (ALG == ALG_SSSP && ROT && a.pol.hub_window)
             ops.hub_hi = (uint64_t)ld_relaxed(&ctl->next_min[slot]) + a.pol.hub_window;
         const uint32_t *bmc = ROT ? a.bm[slot] : a.bm[0];
@@ -1022,22 +1057,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         const uint32_t ntiles = (ws == WS_BM) ? (a.V + BS - 1) / BS : (qn + tile_n - 1) / tile_n;
         const bool hubs = (map == MAP_H) && a.has_hubs;
 
-        if (AG_WARPH && TUNED && map == MAP_H && ws == WS_QU) {
-            // warp-scheduled tiles of tn <= 32 elements (>= 2 tiles per warp), claimed one ahead
-            const uint32_t nwarps = a.nblocks * WARPS_PER_CTA, lane = lane_id();
-            uint32_t tn = (qn + 2 * nwarps - 1) / (2 * nwarps);
-            tn = tn < 1u ? 1u : (tn > 32u ? 32u : tn);
-            const uint32_t nt = (qn + tn - 1) / tn;
-            uint32_t t = blockIdx.x * WARPS_PER_CTA + (threadIdx.x >> 5);
-            while (t < nt) {
-                uint32_t nxt = 0;
-                if (lane == 0) nxt = nwarps + atomicAdd(&ctl->tile_ctr[slot], 1u);
-                const uint32_t i = t * tn + lane;
-                const bool valid = lane < tn && i < qn;
-                process_warp_tile(ops, sm, valid, valid ? qc[i] : 0u, hubs, slot);
-                t = __shfl_sync(0xffffffffu, nxt, 0);
-            }
-        } else {
+        {
             // dynamic tile scheduler: first tile static, then one atomic per tile, fetched one tile ahead
             // (double-buffered in smem; the __syncthreads_or below orders the write before the read)
             uint32_t t = blockIdx.x;
@@ -1066,7 +1086,13 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         ops.warp_flush(true);
         block_reduce_flush(ops, sm, ctl, slot);
         grid_barrier(ctl, a.nblocks);
-        n = ROT ? ld_relaxed(&ctl->q_len[(it + 1) % 3]) : ld_relaxed(&ctl->pend_count);
+        if (ops.freeo) {
+            n = ld_relaxed(&ctl->free_any[(it + 1) % 3]) ? 1u : 0u;   // exact size after the compaction
+            in_raw = true;
+        } else {
+            n = ROT ? ld_relaxed(&ctl->q_len[(it + 1) % 3]) : ld_relaxed(&ctl->pend_count);
+            in_raw = false;
+        }
         prev_ws = ws;
         prev_var = var;
         n_prev = qn;

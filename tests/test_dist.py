@@ -180,3 +180,146 @@ def test_nccl_world1():
         assert np.array_equal(lv, ref) and st.iterations == oracle.bfs_iterations(ref)
     part.free()
     comm.free()
+
+
+# ------------------------------------------------------------------------------------------------
+# Multi-GPU SSSP: same partition, list exchange of (vertex, distance)
+# ------------------------------------------------------------------------------------------------
+def _partitioned_sssp_worker(rank, world, port, scale, src, out_q):
+    """The distributed unordered SSSP of ag_dist_sssp on CPU: every rank relaxes the gathered global
+    list of (u, dist u) over its destination-owned part, then the improved owned vertices are
+    exchanged — all_gather of the counts, then of the (v, dist) lists padded to the largest count."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_lib13_b200 import agraph as A
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    V = 1 << scale
+    b, e = A.owned_range(V, rank, world)
+    part = aggen.rmat_part(scale, 16, 1, b, e)
+    w = aggen.weights(part, seed=2, wmax=100)
+    d = np.full(V, oracle.INF, np.int64)
+    if b <= src < e:
+        d[src] = 0
+    lst = [(src, 0)]
+    rounds = 0
+    while True:
+        improved = set()
+        for u, du in lst:
+            for k in range(part.row_ptr[u], part.row_ptr[u + 1]):
+                v = int(part.col[k])
+                assert b <= v < e
+                nd = du + int(w[k])
+                if nd < d[v]:
+                    d[v] = nd
+                    improved.add(v)
+        mine = sorted(improved)
+        cnt = torch.tensor([len(mine)], dtype=torch.int64)
+        counts = [torch.zeros(1, dtype=torch.int64) for _ in range(world)]
+        dist.all_gather(counts, cnt)
+        maxc = int(max(c.item() for c in counts))
+        rounds += 1
+        if maxc == 0:
+            break
+        buf = torch.full((maxc, 2), -1, dtype=torch.int64)
+        for i, v in enumerate(mine):
+            buf[i, 0], buf[i, 1] = v, int(d[v])
+        bufs = [torch.zeros((maxc, 2), dtype=torch.int64) for _ in range(world)]
+        dist.all_gather(bufs, buf)
+        lst = [(int(v), int(dv)) for t in bufs for v, dv in t.tolist() if v >= 0]
+    out_q.put((rank, b, e, d[b:e].astype(np.uint64).copy(), rounds))
+    dist.destroy_process_group()
+
+
+def test_partitioned_sssp_gloo_world2():
+    import socket
+
+    import torch.multiprocessing as mp
+    scale, world = 9, 2
+    g = aggen.with_weights(aggen.rmat(scale, 16, seed=1), seed=2, wmax=100)
+    src = int(aggen.sources(g, 1)[0])
+    ref, _ = oracle.dijkstra(g, src)
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_partitioned_sssp_worker, args=(r, world, port, scale, src, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(world):
+        item = q.get(timeout=300)
+        res[item[0]] = item
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    d = np.concatenate([res[r][3] for r in range(world)])
+    d = np.where(d == np.uint64(oracle.INF), oracle.INF, d).astype(np.uint32)
+    assert np.array_equal(d, ref)
+    assert res[0][4] == res[1][4]                       # every rank sees the same termination round
+
+
+def _wgraphs():
+    yield aggen.config("C1")
+    yield aggen.random_graph(700, 3000, seed=5)          # directed multigraph with self-loops
+    yield aggen.with_weights(aggen.grid(120, 90))
+    yield aggen.with_weights(aggen.star(20000))          # hub >= HUB_DEG
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world", [1, 2, 3, 5])
+def test_virtual_group_sssp_matches_oracle(world):
+    from paper_conf_ipps_lib13_b200 import agraph as A
+    for g in _wgraphs():
+        comms = A.local_group(world, 0)
+        parts = [A.DistGraph(c, g.V, g.row_ptr, g.col, g.w) for c in comms]
+        for src in sorted(set([0, g.V - 1, int(aggen.sources(g, 1)[0])])):
+            ref, _ = oracle.dijkstra(g, src)
+            d, par, st = A.dist_sssp_group(parts, src, parents=True, stats=True, trace_cap=1 << 14)
+            assert np.array_equal(d, ref), (g.name, world, src)
+            assert oracle.validate(g, src, d, par, weighted=True)[0] == 0
+            assert st.trace_ws[0] == 1 and st.iterations >= 1
+        for p in parts:
+            p.free()
+        for c in comms:
+            c.free()
+
+
+@pytest.mark.gpu
+def test_virtual_group_sssp_local_parts_and_errors():
+    from paper_conf_ipps_lib13_b200 import agraph as A
+    scale, world = 14, 4
+    g = aggen.with_weights(aggen.rmat(scale, 16, seed=1), seed=2, wmax=100)
+    comms = A.local_group(world, 0)
+    parts = []
+    for c in comms:
+        b, e = A.owned_range(g.V, c.rank, world)
+        pg = aggen.rmat_part(scale, 16, 1, b, e)
+        parts.append(A.DistGraph(c, g.V, pg.row_ptr, pg.col, aggen.weights(pg, seed=2, wmax=100), local=True))
+    for src in aggen.sources(g, 3):
+        ref, _ = oracle.dijkstra(g, int(src))
+        d, _, _ = A.dist_sssp_group(parts, int(src))
+        assert np.array_equal(d, ref)
+    # unweighted parts cannot run SSSP
+    uw = [A.DistGraph(c, g.V, g.row_ptr, g.col) for c in A.local_group(2, 0)]
+    with pytest.raises(A.AgError) as e:
+        A.dist_sssp_group(uw, 0)
+    assert e.value.status == "AG_ERR_NO_WEIGHTS"
+
+
+@pytest.mark.gpu
+def test_nccl_world1_sssp():
+    from paper_conf_ipps_lib13_b200 import agraph as A
+    g = aggen.config("C1")
+    uid = A.dist_unique_id()
+    comm = A.Comm.nccl(0, 1, uid, 0)
+    part = A.DistGraph(comm, g.V, g.row_ptr, g.col, g.w)
+    for src in aggen.sources(g, 2):
+        ref, _ = oracle.dijkstra(g, int(src))
+        d, _, st = part.sssp(int(src), stats=True)
+        assert np.array_equal(d, ref)
+    part.free()
+    comm.free()

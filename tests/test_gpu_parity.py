@@ -55,14 +55,15 @@ def pname(p):
            f"{'auto' if not p.workset else A.WS_NAME[p.workset]}_{'paper' if p.kind == 0 else 'tuned'}"
 
 
-def check_bfs(g, G, s, p, expect_level=None):
+def check_bfs(g, G, s, p, expect_level=None, want_parents=True):
     lv, par = oracle.bfs(g, s) if expect_level is None else (expect_level, None)
-    parents = np.empty(g.V, np.uint32)
+    parents = np.empty(g.V, np.uint32) if want_parents else None
     out, _, st = G.bfs(s, parents=parents, policy=p, stats=True, trace_cap=1 << 16)
     assert np.array_equal(out, lv), f"BFS levels differ ({pname(p)}, src {s}): " \
         f"{np.count_nonzero(out != lv)} mismatches"
-    code, bad = oracle.validate(g, s, out, parents, weighted=False)
-    assert code == 0, f"BFS parent certificate failed: {oracle.VALIDATE_MSG[code]} at {bad} ({pname(p)})"
+    if want_parents:
+        code, bad = oracle.validate(g, s, out, parents, weighted=False)
+        assert code == 0, f"BFS parent certificate failed: {oracle.VALIDATE_MSG[code]} at {bad} ({pname(p)})"
     Vr, Er = oracle.reached(g, lv)
     assert (st.reached, st.reached_edges) == (Vr, Er)
     # level-synchronous: ordered AND unordered BFS expand each reached vertex exactly once (16.s43, 26.s33)
@@ -118,6 +119,24 @@ def test_unordered_sssp_window(window):
             for m in (0, 1, 4):
                 check_sssp(g, G, s, pol(0, m, 2 if m else 0, sssp_window=window))
                 check_sssp(g, G, s, pol(0, m, 2 if m else 0, sssp_window=window, sssp_hub_window=1 + window % 5))
+
+
+@pytest.mark.parametrize("free_ppm", [0, 1, 3906, 250000, 1000000])
+def test_free_output_threshold(free_ppm):
+    """Free-output iterations (raw next bitmap by fire-and-forget reductions, compacted by the next
+    iteration) at every threshold: never, always, the default, and in between."""
+    graphs = [aggen.config("C1"), aggen.with_weights(aggen.grid(60, 50), seed=9, wmax=100),
+              aggen.with_weights(aggen.er(5000, 20000, seed=4), seed=5, wmax=100),
+              aggen.with_weights(aggen.star(20000)), aggen.random_graph(300, 1500, seed=3)]
+    for g in graphs:
+        for layout in (0, 1):
+            G = A.Graph.from_csr(g, layout=layout)
+            for s in sorted(set(int(x) for x in aggen.sources(g, 2)) | {0}):
+                for order in (0, 1):
+                    check_bfs(g, G, s, pol(order, free_ppm=free_ppm), want_parents=False)
+                    check_bfs(g, G, s, pol(order, free_ppm=free_ppm))
+                check_sssp(g, G, s, pol(0, free_ppm=free_ppm))
+                check_sssp(g, G, s, pol(0, free_ppm=free_ppm, sssp_window=0, sssp_hub_window=0))
 
 
 @pytest.mark.parametrize("delta", [1, 7, 100, 1000])
@@ -275,6 +294,7 @@ def test_full_size_configs(cfg):
     srcs += [int(s) for s in aggen.sources(g, 2)]
     for s in srcs:
         check_bfs(g, G, s, pol(0))
+        check_bfs(g, G, s, pol(0), want_parents=False)   # bench.py's call: free-output iterations
         check_sssp(g, G, s, pol(0))
         if cfg == "C2":
             check_bfs(g, G, s, pol(0, kind=0))
