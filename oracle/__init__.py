@@ -11,6 +11,9 @@ Contents (each function cites the passage it follows):
                   16.s24; 14.s19; 26.s21).
 * ``dijkstra``  — binary-heap Dijkstra, ``agoracle.c:oracle_dijkstra``
                   (Fig. 5, 18.s28; 14.s20; 22.s10; 26.s36).
+* ``cc``        — min-label connected components, ``agoracle.c:oracle_cc``
+                  (label[v] = min{u : u reaches v}; PAPER.md:10.s9, 12.s13;
+                  SURVEY.md §8(f) NEXT-4; R23).
 * ``validate``  — shortest-path certificate.
 * ``reached``   — V_r, E_r for the byte model.
 * ``selector``  — Fig. 11 decision maker (24.s34-42), see ``oracle/selector.py``.
@@ -60,6 +63,7 @@ def _L():
         _lib.oracle_validate.argtypes = [u32, vp, vp, vp, u32, vp, vp, vp]
         _lib.oracle_reached.argtypes = [u32, vp, vp, vp, vp]
         _lib.oracle_reached.restype = None
+        _lib.oracle_cc.argtypes = [u32, vp, vp, vp]
     return _lib
 
 
@@ -114,6 +118,17 @@ def validate(g, src: int, out: np.ndarray, parent=None, weighted: bool = False):
     rc = _L().oracle_validate(g.V, _p(g.row_ptr), _p(g.col), _p(g.w) if weighted else None, int(src),
                               _p(out), _p(parent), ctypes.addressof(bad))
     return rc, bad.value
+
+
+def cc(g):
+    """label uint32[V]: label[v] = min{u : u reaches v along out-edges} (R23); on a
+    symmetric graph the smallest vertex id of v's connected component."""
+    _chk(g)
+    label = np.empty(g.V, dtype=np.uint32)
+    rc = _L().oracle_cc(g.V, _p(g.row_ptr), _p(g.col), _p(label))
+    if rc != 0:
+        raise ValueError(f"oracle_cc rc={rc}")
+    return label
 
 
 def reached(g, out: np.ndarray):

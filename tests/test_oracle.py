@@ -237,3 +237,43 @@ def test_selector_paper_constants():
     assert selector.block_size(434102, 2 * 16036720) == 64   # CiteSeer avg 73.9 (12.s38) -> 64
     assert selector.block_size(100, 4800) == 64          # avg 48: tie between 32/64 -> up
     assert selector.block_size(100, 100) == 32 and selector.block_size(1, 10**6) == 1024
+
+
+# ---------------------------------------------------------------- min-label CC (NEXT-4)
+def test_cc_closed_forms():
+    """label[v] = min{u : u reaches v} (R23): closed forms."""
+    assert np.array_equal(oracle.cc(aggen.path(17)), np.zeros(17, np.uint32))
+    assert np.array_equal(oracle.cc(aggen.directed_cycle(9)), np.zeros(9, np.uint32))
+    assert np.array_equal(oracle.cc(aggen.star(30)), np.zeros(30, np.uint32))
+    fwd = aggen.csr_from_edges(4, [0, 1, 2], [1, 2, 3])            # 0 -> 1 -> 2 -> 3
+    assert list(oracle.cc(fwd)) == [0, 0, 0, 0]
+    bwd = aggen.csr_from_edges(4, [3, 2, 1], [2, 1, 0])            # 3 -> 2 -> 1 -> 0
+    assert list(oracle.cc(bwd)) == [0, 1, 2, 3]
+    dis = aggen.csr_from_edges(7, [0, 1, 4, 6], [1, 2, 3, 5], symmetrize=True)
+    assert list(oracle.cc(dis)) == [0, 0, 0, 3, 3, 5, 5]
+    loops = aggen.csr_from_edges(3, [1, 1, 2], [1, 1, 2])          # self-loops only
+    assert list(oracle.cc(loops)) == [0, 1, 2]
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_cc_bruteforce_reachability(seed):
+    """Directed multigraphs with self-loops and isolated vertices vs the transitive closure."""
+    rng = np.random.default_rng(500 + seed)
+    V = int(rng.integers(1, 70))
+    M = int(rng.integers(0, 3 * V))
+    g = aggen.random_graph(V, M, seed=500 + seed, wmax=5, sort_rows=bool(seed % 2))
+    lab = oracle.cc(g)
+    assert np.array_equal(lab, bf.reach_min_label(g))
+    assert np.array_equal(lab, bf.jacobi_min_label(g)[0])
+
+
+def test_cc_c1_components():
+    """C1 (symmetric): labels == union-find set minima; one label per component; sizes agree."""
+    g = aggen.config("C1", weighted=False)
+    lab = oracle.cc(g)
+    assert np.array_equal(lab, bf.uf_min_label(g))
+    assert np.array_equal(lab, bf.jacobi_min_label(g)[0])
+    assert np.all(lab <= np.arange(g.V))                     # a vertex reaches itself
+    assert np.all(lab[lab] == lab)                           # a label is its own label
+    sizes = np.bincount(lab, minlength=g.V)[lab]
+    assert np.array_equal(sizes, bf.components(g))
