@@ -398,6 +398,23 @@ def main():
            "sssp_redundancy": statistics.mean(info[step_src(k)][6] / max(1, info[step_src(k)][3]) for k in range(K)),
            "roofline": roof, "gpu_launches": launches, "clocks": sampler.summary()}
 
+    # NEXT-4: min-label connected components on the same graph and engine, timed
+    # separately (not part of the BFS+SSSP step); GTEPS = E / t (every vertex starts in the WS)
+    lab = torch.empty(V, dtype=torch.int32, device="cuda")
+    _, _, sc = G.cc(labels=lab, policy=pol, stats=True)
+    kc = 5
+    evc = [torch.cuda.Event(enable_timing=True) for _ in range(kc + 1)]
+    torch.cuda.synchronize()
+    evc[0].record(stream)
+    for k in range(kc):
+        G.cc(labels=lab, policy=pol, stream=sp)
+        evc[k + 1].record(stream)
+    torch.cuda.synchronize()
+    G.check()
+    tc = statistics.median(evc[k].elapsed_time(evc[k + 1]) for k in range(kc))
+    out["cc"] = {"ms": tc, "gteps": g.E / (tc * 1e-3) / 1e9, "iterations": sc.iterations,
+                 "edges_inspected_per_E": sc.edges_inspected / max(1, g.E), "runs": kc}
+
     # end-to-end through the public API with HOST buffers: CSR upload from pinned memory, both
     # traversals, results read back (the paper's timing scope, 26.s17-18; reading R21)
     if not args.no_e2e:

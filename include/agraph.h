@@ -97,7 +97,10 @@ typedef struct {
                                 elements writes its successor as a raw bitmap with fire-and-forget reductions (no
                                 claiming atomics, no queue appends; BFS without parents only) and the next
                                 iteration converts it to a queue in O(V/32) (the paper's update-vector bitmap,
-                                22.s13-14).  SSSP uses it only on graphs without the degree layout (non-skewed).
+                                22.s13-14).  Used only on graphs without the degree layout (non-skewed; measured
+                                2x slower on R-MAT) unless free_ppm = 1000000 (every iteration, also on
+                                skewed graphs: a diagnostic / test setting).  BFS and ag_cc use t_free from this
+                                field, ag_sssp the same threshold.
                                 0 = never; ag_policy_default: 3906 (V/256) */
     uint32_t reserved;       /* must be 0 */
 } ag_policy;
@@ -198,6 +201,18 @@ ag_status ag_bfs(ag_graph g, uint32_t src, uint32_t *levels, uint32_t *parents, 
  * Errors: as ag_bfs plus AG_ERR_NO_WEIGHTS, AG_ERR_OVERFLOW. */
 ag_status ag_sssp(ag_graph g, uint32_t src, uint32_t *dist, uint32_t *parents, const ag_policy *policy,
                   ag_run_stats *stats, void *stream);
+
+/* Min-label connected components ("other graph algorithms that exhibit
+ * similar computational patterns", PAPER.md:10.s9; connected components, 12.s13; R23):
+ * labels[v] = min{ u : u reaches v along out-edges } (u = v included) in caller ids, i.e. on a
+ * symmetric graph the smallest vertex id of v's connected component.  Same working-set engine as
+ * ag_bfs: WS_0 = every vertex with label = own id; each iteration expands the WS with
+ * atomicMin(label[m], label[n]) and a vertex whose label dropped enters the next WS (Fig. 4 l.8'
+ * with level -> label, no +1), until the WS is empty.  labels: V uint32 (required), host or device.
+ * policy: order must be AG_UNORDERED (AG_ERR_UNSUPPORTED otherwise); mapping / workset / selector
+ * as for ag_bfs.  stats: iterations = label-propagation rounds; reached = V.  Synchronisation as
+ * for ag_bfs.  Errors: AG_ERR_INVALID_ARG, AG_ERR_UNSUPPORTED, AG_ERR_OOM, AG_ERR_CUDA. */
+ag_status ag_cc(ag_graph g, uint32_t *labels, const ag_policy *policy, ag_run_stats *stats, void *stream);
 
 /* Wait for the graph's last enqueued traversal and return its deferred status (AG_OK or
  * AG_ERR_OVERFLOW / AG_ERR_CUDA); clears the deferred status. */

@@ -73,7 +73,7 @@ class RunStats(ctypes.Structure):
 
 
 EXPORTS = ["ag_policy_default", "ag_select", "ag_graph_load_csr", "ag_graph_load_csr_ex", "ag_graph_info_get",
-           "ag_graph_free", "ag_bfs", "ag_sssp", "ag_graph_check", "ag_dist_unique_id", "ag_dist_init",
+           "ag_graph_free", "ag_bfs", "ag_sssp", "ag_cc", "ag_graph_check", "ag_dist_unique_id", "ag_dist_init",
            "ag_dist_init_local", "ag_dist_free", "ag_dist_owned_range", "ag_dist_graph_load_csr",
            "ag_dist_graph_load_local", "ag_dist_bfs", "ag_dist_bfs_group", "ag_dist_sssp", "ag_dist_sssp_group", "ag_set_allocator", "ag_status_string",
            "ag_last_error", "ag_abi_version", "ag_kernel_launches"]
@@ -108,6 +108,7 @@ def lib():
     L.ag_graph_check.argtypes = [vp]
     for f in (L.ag_bfs, L.ag_sssp):
         f.argtypes = [vp, u32, vp, vp, ctypes.POINTER(Policy), ctypes.POINTER(RunStats), vp]
+    L.ag_cc.argtypes = [vp, vp, ctypes.POINTER(Policy), ctypes.POINTER(RunStats), vp]
     L.ag_dist_unique_id.argtypes = [vp]
     L.ag_dist_init.argtypes = [i32, i32, vp, i32, ctypes.POINTER(vp)]
     L.ag_dist_free.argtypes = [vp]
@@ -242,6 +243,13 @@ class Graph:
              trace_cap: int = 0, stream: Optional[int] = None):
         """ag_sssp; returns (dist, parents, Stats|None)."""
         return self._run(lib().ag_sssp, src, dist, parents, policy, stats, trace_cap, stream)
+
+    def cc(self, labels=None, policy: Optional[Policy] = None, stats: bool = False, trace_cap: int = 0,
+           stream: Optional[int] = None):
+        """ag_cc (min-label components, R23); returns (labels, None, Stats|None)."""
+        def fn(h, _src, out, _par, pol, st, strm):
+            return lib().ag_cc(h, out, pol, st, strm)
+        return self._run(fn, 0, labels, None, policy, stats, trace_cap, stream)
 
     def check(self):
         _check(lib().ag_graph_check(self.h))

@@ -303,10 +303,16 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
     d.t2_tuned = 65536;
     d.t_free = (p.kind == AG_POLICY_TUNED && p.free_ppm) ? ((uint64_t)g.V * p.free_ppm + 999999ull) / 1000000ull : ~0ull;
     if (d.t_free == 0) d.t_free = 1;
+    const uint64_t t_free_any = d.t_free;
+    // BFS: free output only on non-skewed graphs too (measured over 32 sources, profiles/r01_free_output_ab.txt:
+    // R-MAT s22 median 0.571 ms without vs 1.19 ms with — during a free-output level the visited bitmap is
+    // not updated, so every edge into a vertex discovered in the same level issues a red.or, tens of millions
+    // on the big R-MAT level; ER n=2^25 6.41 -> 3.69 ms with it)
+    if (g.info.layout == AG_LAYOUT_DEGREE && !(p.free_ppm >= 1000000u)) d.t_free = ~0ull;
     // SSSP: free output only on non-skewed graphs (measured: ER n=2^25 21.4 -> 12.4 ms; R-MAT s22
     // 1.59 -> 2.19 ms, the fire-and-forget red.min on power-law hot targets loses to the claiming
     // atomicMin whose result gates the next-bitmap update)
-    d.t_free_sssp = g.info.layout == AG_LAYOUT_DEGREE ? ~0ull : d.t_free;
+    d.t_free_sssp = (g.info.layout == AG_LAYOUT_DEGREE && !(p.free_ppm >= 1000000u)) ? ~0ull : t_free_any;
     return d;
 }
 
@@ -347,8 +353,8 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
     attrs[0].id = cudaLaunchAttributeCooperative;
     attrs[0].val.cooperative = 1;
     int nattr = 1;
-    void *wbase = ALG == ALG_SSSP ? (void *)a.P : (void *)a.vis;
-    size_t wbytes = ALG == ALG_SSSP ? (size_t)g->V * 8 : (size_t)g->nwords * 4;
+    void *wbase = ALG == ALG_SSSP ? (void *)a.P : ALG == ALG_CC ? (void *)a.level : (void *)a.vis;
+    size_t wbytes = ALG == ALG_SSSP ? (size_t)g->V * 8 : ALG == ALG_CC ? (size_t)g->V * 4 : (size_t)g->nwords * 4;
     if (g->persist_bytes > 0 && getenv("AG_NO_L2_WINDOW") == nullptr) {
         if (wbytes > g->max_window) wbytes = g->max_window;
         attrs[1].id = cudaLaunchAttributeAccessPolicyWindow;
@@ -418,7 +424,7 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
     a.ctl = (Ctl *)g->d_ctl;
     a.perm = g->d_perm;
     a.inv = g->d_inv;
-    if (alg == ALG_BFS) {
+    if (alg != ALG_SSSP) {   // BFS levels / CC labels
         if (g->d_inv) {  // traverse in the degree layout, gather back to caller ids at the end
             if (!g->d_level && (s = dev_alloc((void **)&g->d_level, (size_t)g->V * 4 + 128, g->device)) != AG_OK) return s;
             if (d_par && !g->d_lpar && (s = dev_alloc((void **)&g->d_lpar, (size_t)g->V * 4 + 128, g->device)) != AG_OK)
@@ -446,7 +452,7 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
     a.pol = resolve_policy(pol, *g);
     a.src = src;
     a.epoch = ++g->epoch;
-    a.max_iters = alg == ALG_BFS ? g->V + 2 : 4u * g->V + 64u;
+    a.max_iters = alg != ALG_SSSP ? g->V + 2 : 4u * g->V + 64u;   // CC: <= longest min-label chain + 1
     if (a.max_iters < g->V) a.max_iters = 0xFFFFFFF0u;
     a.has_hubs = g->info.max_deg >= HUB_DEG;
 
@@ -456,6 +462,9 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
     if (alg == ALG_BFS) {
         s = (pol.order == AG_ORDERED) ? launch_traverse<ALG_BFS, ORD_O, Off>(g, a, st)
                                       : launch_traverse<ALG_BFS, ORD_U, Off>(g, a, st);
+    } else if (alg == ALG_CC) {
+        if (pol.order == AG_ORDERED) return set_error(AG_ERR_UNSUPPORTED, "ag_cc is unordered only (DESIGN.md R23)");
+        s = launch_traverse<ALG_CC, ORD_U, Off>(g, a, st);
     } else {
         s = (pol.order == AG_ORDERED) ? launch_traverse<ALG_SSSP, ORD_O, Off>(g, a, st)
                                       : launch_traverse<ALG_SSSP, ORD_U, Off>(g, a, st);
@@ -785,6 +794,7 @@ ag_status ag_graph_check(ag_graph g) {
 static ag_status query(ag_graph g, int alg, uint32_t src, uint32_t *out, uint32_t *parents, const ag_policy *p,
                        ag_run_stats *stats, void *stream) {
     if (!g || !out) return set_error(AG_ERR_INVALID_ARG, "NULL argument");
+    if (alg == ALG_CC && parents) return set_error(AG_ERR_INVALID_ARG, "ag_cc has no parents");
     if (src >= g->V) return set_error(AG_ERR_SRC_RANGE, "src %u >= V %u", src, g->V);
     if (alg == ALG_SSSP && !g->d_cw) return set_error(AG_ERR_NO_WEIGHTS, "graph was loaded without weights");
     if (g->dist) return set_error(AG_ERR_INVALID_ARG, "distributed graph: use ag_dist_bfs");
@@ -801,6 +811,10 @@ ag_status ag_bfs(ag_graph g, uint32_t src, uint32_t *levels, uint32_t *parents, 
 ag_status ag_sssp(ag_graph g, uint32_t src, uint32_t *dist, uint32_t *parents, const ag_policy *policy,
                   ag_run_stats *stats, void *stream) {
     return query(g, ALG_SSSP, src, dist, parents, policy, stats, stream);
+}
+
+ag_status ag_cc(ag_graph g, uint32_t *labels, const ag_policy *policy, ag_run_stats *stats, void *stream) {
+    return query(g, ALG_CC, 0, labels, nullptr, policy, stats, stream);
 }
 
 }  // extern "C"

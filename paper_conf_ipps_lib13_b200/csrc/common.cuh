@@ -46,7 +46,7 @@ constexpr uint32_t INF = 0xFFFFFFFFu;
 constexpr unsigned long long INF64 = 0xFFFFFFFFFFFFFFFFull;
 constexpr uint32_t MAX_FINITE = 0xFFFFFFFEu;
 
-enum { ALG_BFS = 0, ALG_SSSP = 1 };
+enum { ALG_BFS = 0, ALG_SSSP = 1, ALG_CC = 2 };   // CC: min-label components (NEXT-4, R23)
 enum { ORD_U = 0, ORD_O = 1 };
 enum { MAP_T = 1, MAP_W = 2, MAP_B = 3, MAP_H = 4 };
 enum { WS_BM = 1, WS_QU = 2 };
@@ -220,6 +220,9 @@ __device__ __forceinline__ uint32_t ld_ro(const uint32_t *p) { return __ldg(p); 
 __device__ __forceinline__ unsigned long long ld_ro(const unsigned long long *p) { return __ldg(p); }
 __device__ __forceinline__ void red_or(uint32_t *p, uint32_t v) {
     asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void red_min32(uint32_t *p, uint32_t v) {
+    asm volatile("red.relaxed.gpu.global.min.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 __device__ __forceinline__ void red_min64(unsigned long long *p, unsigned long long v) {
     asm volatile("red.relaxed.gpu.global.min.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");

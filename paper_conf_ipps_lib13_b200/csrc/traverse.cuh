@@ -13,6 +13,8 @@
 //           SSSP unordered : packed 64-bit atomicMin((dist<<32)|parent)        (Fig. 5 l.6-9)
 //           SSSP ordered   : bucket [lo, lo+delta) of the pending set; lo = findmin by block
 //                            reduction + atomicMin fused into the pass         (Fig. 5; 22.s9-11)
+//           CC (NEXT-4)    : atomicMin(label[v], label[u]), "if (m.label > n.label)": Fig. 4 l.8'
+//                            with level -> label and no +1; WS_0 = every vertex (R23)
 //     a5  the next working set is written as the update vector = next-frontier bitmap (atomicOr,
 //         20.s39-40) AND as a queue by warp-aggregated atomic append (22.s18), so either
 //         representation is ready for the next iteration without an extra pass.
@@ -49,7 +51,7 @@ struct TravArgs {
     const uint2 *cw;            // SSSP: interleaved (col, w)
     uint32_t V;
     uint32_t nwords;
-    uint32_t *level;            // BFS level array (V), in device-layout ids
+    uint32_t *level;            // BFS level array / CC label array (V), in device-layout ids
     uint32_t *parent;           // BFS parent array (V) or nullptr, in device-layout ids
     const uint32_t *perm;       // degree layout: new id -> caller id (nullptr = identity layout)
     const uint32_t *inv;        //                caller id -> new id
@@ -144,6 +146,8 @@ struct Ops {
         bool ex = true;
         if constexpr (ALG == ALG_BFS) {
             uval = it;  // the frontier of iteration it is exactly level it (level-synchronous, 26.s33)
+        } else if constexpr (ALG == ALG_CC) {
+            uval = ld_relaxed(&a.level[u]);   // the current label (never above the one that queued u)
         } else if (a.ulist) {
             // listed entry: uval (the sender's distance of u) was set by the caller; every entry expands
         } else {
@@ -205,7 +209,9 @@ struct Ops {
             uval = e.y;
         } else {
             u = key;
-            uval = (ALG == ALG_BFS) ? it : (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
+            uval = (ALG == ALG_BFS) ? it
+                 : (ALG == ALG_CC)  ? ld_relaxed(&a.level[u])
+                                    : (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
         }
     }
 
@@ -215,6 +221,7 @@ struct Ops {
     using St = uint32_t;
     __device__ __forceinline__ St status(uint32_t v) const {
         if constexpr (ALG == ALG_SSSP) return (uint32_t)(ld_keep(a.P + v, pol_keep) >> 32);
+        else if constexpr (ALG == ALG_CC) return ld_keep(a.level + v, pol_keep);   // label[v]
         else return ld_keep(a.vis + (v >> 5), pol_keep);   // BFS: visited bit (level-synchronous: set <=> level <= current+1)
     }
 
@@ -224,7 +231,10 @@ struct Ops {
         const uint32_t m = 1u << (v & 31);
         bool nw = false;
         if (!valid) return false;
-        if constexpr (ALG == ALG_BFS) {
+        if constexpr (ALG == ALG_CC) {
+            if (s > uval && atomicMin(&a.level[v], uval) > uval)          // m.label > n.label
+                nw = !(atomicOr(bm_next + (v >> 5), m) & m);               // ws.add(m), deduped
+        } else if constexpr (ALG == ALG_BFS) {
             const uint32_t nl = uval + 1;
             if constexpr (ORD == ORD_O) {
                 if (!(s & m)) {                                        // m.level == INF ?   (Fig. 4 l.8)
@@ -285,6 +295,9 @@ struct Ops {
             if constexpr (ALG == ALG_BFS) {
                 nd[j] = 0;
                 if (ok[j] && !((st[j] >> (v[j] & 31)) & 1u)) cm |= 1u << j;   // m.level == INF / > level
+            } else if constexpr (ALG == ALG_CC) {
+                nd[j] = uv[j];
+                if (ok[j] && st[j] > uv[j]) cm |= 1u << j;                      // m.label > n.label
             } else {
                 nd[j] = (uint64_t)uv[j] + wt[j];                                // d = n.distance + w (l.6)
                 if (ok[j]) {
@@ -304,6 +317,8 @@ struct Ops {
                     if constexpr (ALG == ALG_SSSP) {
                         red_min64(&a.P[v[j]], (nd[j] << 32) | u[j]);            // m.distance = d (l.8)
                         vmin = min(vmin, (uint32_t)nd[j]);
+                    } else if constexpr (ALG == ALG_CC) {
+                        red_min32(&a.level[v[j]], uv[j]);                       // m.label = n.label
                     }
                     red_or(bm_next + (v[j] >> 5), 1u << (v[j] & 31));           // ws.add(m)       (l.9)
                 }
@@ -312,7 +327,20 @@ struct Ops {
             return 0u;
         }
         uint32_t nwm = 0;
-        if constexpr (ALG == ALG_BFS) {
+        if constexpr (ALG == ALG_CC) {
+            uint32_t r[NB];
+#pragma unroll
+            for (int j = 0; j < NB; ++j) r[j] = ((cm >> j) & 1u) ? atomicMin(&a.level[v[j]], uv[j]) : 0u;
+            uint32_t ob[NB];
+#pragma unroll
+            for (int j = 0; j < NB; ++j) {
+                ob[j] = 0u;
+                if (((cm >> j) & 1u) && r[j] > uv[j]) ob[j] = atomicOr(bm_next + (v[j] >> 5), 1u << (v[j] & 31));
+            }
+#pragma unroll
+            for (int j = 0; j < NB; ++j)   // lowered AND first to set the bit: ws.add(m), deduped
+                if (((cm >> j) & 1u) && r[j] > uv[j] && !(ob[j] & (1u << (v[j] & 31)))) nwm |= 1u << j;
+        } else if constexpr (ALG == ALG_BFS) {
             // (2) every claiming atomic of the batch issued back to back, (3) results resolved
             uint32_t r[NB];
 #pragma unroll
@@ -930,13 +958,19 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             a.level[v] = (v == src) ? 0u : INF;
             if (a.parent) a.parent[v] = (v == src) ? src : INF;
         }
+    } else if (ALG == ALG_CC) {   // label = own (caller) id; WS_0 = every vertex, as queue and as bitmap
+        for (uint32_t v = gtid; v < a.V; v += gthreads) {
+            a.level[v] = a.perm ? a.perm[v] : v;
+            a.q[0][v] = v;
+        }
     } else {
         for (uint32_t v = gtid; v < a.V; v += gthreads)
             a.P[v] = (v == src) ? (unsigned long long)src : INF64;   // dist 0, parent src
     }
     const uint32_t sbit = 1u << (src & 31), sword = src >> 5;
     for (uint32_t wi = gtid; wi < a.nwords; wi += gthreads) {
-        a.bm[0][wi] = (wi == sword) ? sbit : 0u;
+        a.bm[0][wi] = (ALG == ALG_CC) ? ((wi + 1 < a.nwords || (a.V & 31) == 0) ? ~0u : (1u << (a.V & 31)) - 1u)
+                                      : ((wi == sword) ? sbit : 0u);
         if (ROT) {
             a.bm[1][wi] = 0u;
             a.bm[2][wi] = 0u;
@@ -944,9 +978,9 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         if (ALG == ALG_BFS) a.vis[wi] = (wi == sword) ? sbit : 0u;
     }
     if (gtid == 0) {
-        a.q[0][0] = src;
+        if (ALG != ALG_CC) a.q[0][0] = src;
         for (int s = 0; s < 3; ++s) {
-            ctl->q_len[s] = (s == 0) ? 1u : 0u;
+            ctl->q_len[s] = (s == 0) ? (ALG == ALG_CC ? a.V : 1u) : 0u;
             ctl->next_min[s] = (s == 0) ? 0u : INF;
             ctl->tile_ctr[s] = 0;
             ctl->hub_tail[s] = 0;
@@ -963,7 +997,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         ctl->eexp = 0;
     }
     grid_barrier(ctl, a.nblocks);
-    uint32_t n = 1;   // |WS_0| = |{src}|
+    uint32_t n = (ALG == ALG_CC) ? a.V : 1u;   // |WS_0| = |{src}| (CC: every vertex)
 
     uint32_t prev_ws = WS_QU;   // representation used in the previous iteration
     uint8_t prev_var = 0;
@@ -1038,8 +1072,8 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         Ops<ALG, ORD, Off> ops(a, it, hi, append);
         ops.wbuf = sm.wq[threadIdx.x >> 5];
         // free output (tuned, unordered, big working sets; BFS only without parents: a claim decides them)
-        ops.freeo = TUNED && ROT && (ALG == ALG_SSSP ? (uint64_t)qn >= a.pol.t_free_sssp
-                                                     : ((uint64_t)qn >= a.pol.t_free && a.parent == nullptr));
+        ops.freeo = TUNED && ROT && (ALG != ALG_BFS ? (uint64_t)qn >= a.pol.t_free_sssp
+                                                    : ((uint64_t)qn >= a.pol.t_free && a.parent == nullptr));
         if (ALG == ALG_SSSP && ROT && a.pol.hub_window)
             ops.hub_hi = (uint64_t)ld_relaxed(&ctl->next_min[slot]) + a.pol.hub_window;
         const uint32_t *bmc = ROT ? a.bm[slot] : a.bm[0];
@@ -1114,7 +1148,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
                 a.parent_out[v] = (pv == INF64) ? INF : (a.perm ? a.perm[pp] : pp);
             }
         }
-    } else if (a.inv) {     // BFS in the degree layout: gather back to caller ids
+    } else if (a.inv) {     // BFS / CC in the degree layout: gather back to caller ids
         for (uint32_t v = gtid; v < a.V; v += gthreads) {
             const uint32_t i = a.inv[v];
             a.out_level[v] = a.level[i];

@@ -24,17 +24,33 @@ def main():
     ap.add_argument("--workset", type=int, default=0)
     ap.add_argument("--kind", type=int, default=1)
     ap.add_argument("--delta", type=int, default=1)
+    ap.add_argument("--set", action="append", default=[], help="policy field=value")
+    ap.add_argument("--summary", action="store_true", help="print one median line (skips the first query)")
     args = ap.parse_args()
-    g = aggen.config(args.config)
-    G = A.Graph.from_csr(g)
+    g = aggen.config(args.config, weighted=args.alg == "sssp")
+    G = A.Graph.from_csr(g, weighted=args.alg == "sssp")
     p = A.policy_default(0)
     p.order, p.mapping, p.workset, p.kind, p.delta = args.order, args.mapping, args.workset, args.kind, args.delta
+    for kv in args.set:
+        k, v = kv.split("=")
+        setattr(p, k, int(v))
     srcs = aggen.sources(g, 64, seed=3)
+    ms = []
     for k in range(args.n):
-        fn = G.bfs if args.alg == "bfs" else G.sssp
-        _, _, st = fn(int(srcs[k % 64]), policy=p, stats=True)
-        print(f"{args.alg} src={int(srcs[k % 64])} ms={st.device_ms:.3f} iters={st.iterations} "
-              f"Er={st.reached_edges} GTEPS={st.reached_edges / st.device_ms / 1e6:.1f}", flush=True)
+        if args.alg == "cc":
+            _, _, st = G.cc(policy=p, stats=True)
+        else:
+            fn = G.bfs if args.alg == "bfs" else G.sssp
+            _, _, st = fn(int(srcs[k % 64]), policy=p, stats=True)
+        ms.append(st.device_ms)
+        if not args.summary:
+            print(f"{args.alg} src={int(srcs[k % 64])} ms={st.device_ms:.3f} iters={st.iterations} "
+                  f"Er={st.reached_edges} GTEPS={st.reached_edges / st.device_ms / 1e6:.1f}", flush=True)
+    if args.summary:
+        import statistics
+        t = ms[1:] if len(ms) > 1 else ms
+        print(f"{args.config} {args.alg} {' '.join(args.set)} n={len(t)} median_ms={statistics.median(t):.3f} "
+              f"mean_ms={statistics.mean(t):.3f} max_ms={max(t):.3f}", flush=True)
 
 
 if __name__ == "__main__":
