@@ -340,6 +340,31 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
     int occ = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, BS, dyn);
     if (e != cudaSuccess || occ < 1) return cuda_status(e == cudaSuccess ? cudaErrorLaunchOutOfResources : e, "occupancy");
+    // L1/shared carveout: request just the shared memory the resident CTAs need so the rest of the
+    // 256 KB goes to L1, where the status gathers hit (the driver otherwise picked a 132 KB shared
+    // configuration for ~100 KB of use).  Once per kernel; AG_CARVEOUT=<pct> or -1 overrides.
+    static int carved[2] = {0, 0};   // per specialisation (tuned / paper variants)
+    if (!carved[tuned]) {
+        carved[tuned] = 1;
+        int pct = -1;
+        const char *ev = getenv("AG_CARVEOUT");
+        cudaFuncAttributes fa;
+        if (ev) {
+            pct = atoi(ev);
+        } else if (cudaFuncGetAttributes(&fa, fn) == cudaSuccess) {
+            const double need = (double)occ * ((double)fa.sharedSizeBytes + dyn + 1024.0);
+            pct = (int)((need * 100.0 + 228.0 * 1024.0 - 1.0) / (228.0 * 1024.0));
+            if (pct > 100) pct = 100;
+        }
+        if (pct >= 0) {
+            cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+            int occ2 = 0;
+            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, fn, BS, dyn) != cudaSuccess || occ2 < occ) {
+                cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, -1);   // keep occupancy
+            }
+        }
+        cudaGetLastError();
+    }
     a.nblocks = (uint32_t)(occ * g->num_sms);
     // Cooperative launch (co-resident grid for the software grid barrier) with an L2 access-policy
     // window marking the per-vertex status array persisting, so the ~1 GB CSR stream does not evict

@@ -203,7 +203,7 @@ __global__ void popcount_kernel(const uint32_t *bm, uint32_t nwords, unsigned lo
 template <typename Off>
 __global__ void __launch_bounds__(BS, AG_MINB_BFS) dist_level_kernel(const TravArgs<Off> a, uint32_t L,
                                                                      const uint32_t *front) {
-    __shared__ TileSmem<Off> sm;
+    __shared__ TileSmem<Off, wq_cap<ALG_BFS>()> sm;
     Ctl *ctl = a.ctl;
     const uint32_t slot = 0;
     const uint32_t gtid = blockIdx.x * BS + threadIdx.x, gthreads = a.nblocks * BS;
@@ -240,7 +240,7 @@ __global__ void __launch_bounds__(BS, AG_MINB_BFS) dist_level_kernel(const TravA
 template <typename Off>
 __global__ void __launch_bounds__(BS, AG_MINB_SSSP) dist_sssp_kernel(const TravArgs<Off> a, const uint2 *list,
                                                                      uint32_t n) {
-    __shared__ TileSmem<Off> sm;
+    __shared__ TileSmem<Off, wq_cap<ALG_SSSP>()> sm;
     Ctl *ctl = a.ctl;
     const uint32_t slot = 0;
     Ops<ALG_SSSP, ORD_U, Off> ops(a, 0, ~0ull, true);   // it 0: next bitmap bm[1], next queue q[1]

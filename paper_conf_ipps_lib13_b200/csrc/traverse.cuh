@@ -82,10 +82,15 @@ struct TravArgs {
 };
 
 // per-warp staging capacity: one batch appends at most 32 x (edges per thread per batch), plus < 32 left over
-constexpr int BATCH_MAX = (EB_MAX > 4 * AG_QB) ? EB_MAX : 4 * AG_QB;
-constexpr int WQ_CAP = 32 * BATCH_MAX + 32;
+// (sized per algorithm: the smaller SSSP buffer lets the L1/shared carveout leave more L1 to the status
+// gathers, see launch_traverse)
+template <int ALG>
+constexpr int wq_cap() {
+    return 32 * ((ALG == ALG_SSSP) ? (AG_EB_SSSP > 2 * AG_QB_SSSP ? AG_EB_SSSP : 2 * AG_QB_SSSP)
+                                   : (AG_EB_BFS > 4 * AG_QB ? AG_EB_BFS : 4 * AG_QB)) + 32;
+}
 
-template <typename Off>
+template <typename Off, int WQ_CAP>
 struct __align__(16) TileSmem {
     Off beg[BS];
     uint32_t u[BS];
@@ -593,8 +598,8 @@ struct Ops {
 };
 
 // ------------------------------------------------------------------------------------------------
-template <int ALG, int ORD, typename Off>
-__device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, TileSmem<Off> &sm, Ctl *ctl,
+template <int ALG, int ORD, typename Off, typename SmT>
+__device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, SmT &sm, Ctl *ctl,
                                                    uint32_t slot) {
     const unsigned lane = lane_id(), wid = threadIdx.x >> 5;
     unsigned long long ne = warp_sum(ops.ne), nv = warp_sum(ops.nv);
@@ -641,8 +646,8 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, Tile
 // ------------------------------------------------------------------------------------------------
 // One tile: thread tid holds working-set element (valid, u).  Applies the mapping.
 // ------------------------------------------------------------------------------------------------
-template <bool TUNED, int ALG, int ORD, typename Off>
-__device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, TileSmem<Off> &sm, uint32_t map,
+template <bool TUNED, int ALG, int ORD, typename Off, typename SmT>
+__device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, SmT &sm, uint32_t map,
                                              bool valid, uint32_t u, uint32_t group, bool hubs, uint32_t slot,
                                              uint32_t uval_in = 0, uint32_t key = 0xFFFFFFFFu) {
     const TravArgs<Off> &a = ops.a;
@@ -793,8 +798,8 @@ __device__ __forceinline__ unsigned long long hub_wait(const TravArgs<Off> &a, u
 // drain the hub-chunk tasks of this iteration (hybrid mapping).  Thread 0 runs two claims ahead and
 // loads the next task word before the CTA expands the current one, so in steady state the claim and
 // fetch latency hides behind the expansion; tasks reach the CTA through two shared-memory slots.
-template <int ALG, int ORD, typename Off>
-__device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, TileSmem<Off> &sm, uint32_t slot) {
+template <int ALG, int ORD, typename Off, typename SmT>
+__device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, SmT &sm, uint32_t slot) {
     const TravArgs<Off> &a = ops.a;
     Ctl *ctl = a.ctl;
     __syncthreads();
@@ -862,8 +867,8 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, TileSmem<Off
 // takes one word per step, one atomic per CTA step.  BFS keeps only the unvisited bits, marks them
 // visited and assigns their level (the bitmap held candidates, not claims); SSSP keeps every bit.
 // Every word is cleared for reuse.
-template <int ALG, typename Off>
-__device__ __forceinline__ void compact_raw(const TravArgs<Off> &a, TileSmem<Off> &sm, uint32_t *bm, uint32_t lvl,
+template <int ALG, typename Off, typename SmT>
+__device__ __forceinline__ void compact_raw(const TravArgs<Off> &a, SmT &sm, uint32_t *bm, uint32_t lvl,
                                             uint32_t *q, unsigned *qlen) {
     const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
     for (uint32_t w0 = blockIdx.x * BS; w0 < a.nwords; w0 += a.nblocks * BS) {
@@ -945,7 +950,7 @@ template <int ALG, int ORD, typename Off, bool TUNED>
 __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T : AG_MINB_SSSP)
                                                       : (TUNED ? AG_MINB_BFS_T : AG_MINB_BFS))
     traverse_kernel(const TravArgs<Off> a) {
-    __shared__ TileSmem<Off> sm;
+    __shared__ TileSmem<Off, wq_cap<ALG>()> sm;
 
     Ctl *ctl = a.ctl;
     const uint32_t gtid = blockIdx.x * BS + threadIdx.x, gthreads = a.nblocks * BS;
