@@ -100,6 +100,16 @@ struct alignas(128) Ctl {
     unsigned int iterations;
     unsigned int aborted;             // iteration cap hit (never expected)
     unsigned long long vexp, eexp;    // totals
+    // small-frontier mode (tuned kernels): CTAs >= small_ctas park while |WS| < t_small and are woken
+    // with the iteration to resume at (wake_n = 0: terminate).  Own 128-B line: the parked CTAs poll
+    // it, and must not slow the atomics on the per-iteration counters above.
+    alignas(128) unsigned int wake_gen;   // wake events so far (monotone across launches)
+    unsigned int wake_it, wake_n, wake_nprev;
+    unsigned int pad2[28];
+    // virtual CTA numbering (small-frontier mode): one "leader" CTA per SM gets vid [0, leaders), the
+    // others [leaders, nblocks); counters double-buffered by launch parity (the other half is zeroed)
+    unsigned int sm_rank[256];        // CTAs that have arrived on SM s (mod CTAs per SM = rank on s)
+    unsigned int lead_cnt[2], other_cnt[2];
 };
 
 // Policy as seen by the device (plain integers; filled from ag_policy on the host).
@@ -121,6 +131,8 @@ struct DevPolicy {
     uint32_t t2_tuned;    // tuned policy: thread mapping below this |WS| on low-degree graphs
     uint64_t t_free;      // tuned policy: free (raw-bitmap) output from this |WS| on (~0 = never), BFS
     uint64_t t_free_sssp; //   ... SSSP (never on skewed graphs: red.min on hot targets loses, tools/gpu_free_ab.sh)
+    uint32_t small_ctas;  // tuned kernels: CTAs that run an iteration whose |WS| < t_small (the rest park)
+    uint32_t t_small;     //   0 = off
 };
 
 // The decision maker.  PAPER: Fig. 11 with readings R12/R13:
@@ -292,10 +304,11 @@ __device__ __forceinline__ unsigned atom_add_acqrel(unsigned *p, unsigned v) {
 // CTA 0 adds 0x80000000 - (nblocks - 1), every other CTA adds 1, so the top bit flips exactly when
 // the last CTA arrives; everyone spins on that bit (measured on B200: ~1.6 us at 592 CTAs, faster
 // than a two-level tree with a separate release word).  Self-resetting across launches.
-__device__ __forceinline__ void grid_barrier(Ctl *ctl, unsigned nblocks) {
+// `first`: exactly one participating CTA passes true (default: CTA 0).
+__device__ __forceinline__ void grid_barrier(Ctl *ctl, unsigned nblocks, bool first) {
     __syncthreads();
     if (threadIdx.x == 0) {
-        const unsigned inc = (blockIdx.x == 0) ? (0x80000000u - (nblocks - 1)) : 1u;
+        const unsigned inc = first ? (0x80000000u - (nblocks - 1)) : 1u;
         __threadfence();
         const unsigned old = atomicAdd(&ctl->bar_count, inc);
         while (((old ^ ld_relaxed(&ctl->bar_count)) & 0x80000000u) == 0) {
@@ -304,6 +317,7 @@ __device__ __forceinline__ void grid_barrier(Ctl *ctl, unsigned nblocks) {
     }
     __syncthreads();
 }
+__device__ __forceinline__ void grid_barrier(Ctl *ctl, unsigned nblocks) { grid_barrier(ctl, nblocks, blockIdx.x == 0); }
 
 // Warp-aggregated append of v (where flag) to a queue: one atomic per warp-step ("each thread uses an
 // atomic operation only to get a unique insertion index", 22.s18, aggregated per warp).

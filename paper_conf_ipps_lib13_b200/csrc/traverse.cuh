@@ -135,6 +135,7 @@ struct Ops {
     bool ovf;
     bool freeo = false;     // free output: next working set = raw bitmap by fire-and-forget reductions
     bool any = false;       //   ... and this thread set at least one bit of it
+    uint32_t nact = 0;      // CTAs taking part in this iteration
 
     __device__ Ops(const TravArgs<Off> &a_, uint32_t it_, uint64_t hi_, bool append_)
         : a(a_), it(it_), hi(hi_), append_next(append_), fenced(ALG == ALG_SSSP && ORD == ORD_O && a_.pol.delta > 1),
@@ -776,7 +777,7 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, SmT &sm, u
 // Wait for hub task t of this iteration: its word, or 0 once the producers are all done and t is
 // past the final tail (thread 0 only).
 template <typename Off>
-__device__ __forceinline__ unsigned long long hub_wait(const TravArgs<Off> &a, uint32_t t, uint32_t slot) {
+__device__ __forceinline__ unsigned long long hub_wait(const TravArgs<Off> &a, uint32_t t, uint32_t slot, uint32_t nact) {
     Ctl *ctl = a.ctl;
     if (t >= a.hub_cap) return 0ull;   // overflow (flagged by the producer)
     for (;;) {
@@ -786,7 +787,7 @@ __device__ __forceinline__ unsigned long long hub_wait(const TravArgs<Off> &a, u
             __nanosleep(32);
             continue;
         }
-        if (ld_relaxed(&ctl->stage_done[slot]) == a.nblocks) {
+        if (ld_relaxed(&ctl->stage_done[slot]) == nact) {
             (void)ld_acquire(&ctl->stage_done[slot]);   // every producer's tail reservation is visible
             if (t < ld_relaxed(&ctl->hub_tail[slot])) continue;
             return 0ull;
@@ -810,7 +811,7 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, SmT &sm, uin
         atomicAdd(&ctl->stage_done[slot], 1u);
         const uint32_t c0 = atomicAdd(&ctl->hub_head[slot], 1u);
         c1 = atomicAdd(&ctl->hub_head[slot], 1u);
-        const unsigned long long w = hub_wait(a, c0, slot);
+        const unsigned long long w = hub_wait(a, c0, slot, ops.nact);
         if (w) {
             a.hub[c0] = 0ull;
             pre = c1 < a.hub_cap ? ld_relaxed64(a.hub + c1) : 0ull;
@@ -848,7 +849,7 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, SmT &sm, uin
             ops.template pieces<QB>(pu, pv, pq, plo, phi, pok);
         }
         if (threadIdx.x == 0) {
-            const unsigned long long wn = pre ? pre : hub_wait(a, c1, slot);
+            const unsigned long long wn = pre ? pre : hub_wait(a, c1, slot, ops.nact);
             if (wn) {
                 a.hub[c1] = 0ull;
                 c1 = c2;
@@ -869,9 +870,9 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, SmT &sm, uin
 // Every word is cleared for reuse.
 template <int ALG, typename Off, typename SmT>
 __device__ __forceinline__ void compact_raw(const TravArgs<Off> &a, SmT &sm, uint32_t *bm, uint32_t lvl,
-                                            uint32_t *q, unsigned *qlen) {
+                                            uint32_t *q, unsigned *qlen, uint32_t nact, uint32_t vid) {
     const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
-    for (uint32_t w0 = blockIdx.x * BS; w0 < a.nwords; w0 += a.nblocks * BS) {
+    for (uint32_t w0 = vid * BS; w0 < a.nwords; w0 += nact * BS) {
         const uint32_t wi = w0 + threadIdx.x;
         uint32_t word = wi < a.nwords ? bm[wi] : 0u;
         if (word) {
@@ -1001,8 +1002,30 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         ctl->vexp = 0;
         ctl->eexp = 0;
     }
+    // small-frontier mode: wake events seen so far (read before the barrier: no wake can precede it),
+    // and the virtual CTA id: one leader per SM first, so a small iteration runs on every SM
+    uint32_t wgen = ld_relaxed(&ctl->wake_gen);
+    const uint32_t lpar = a.epoch & 1u;
+    if (threadIdx.x == 0) {
+        uint32_t smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        const uint32_t per_sm = a.pol.small_ctas ? (a.nblocks + a.pol.small_ctas - 1) / a.pol.small_ctas : 1u;
+        const bool leader = atomicAdd(&ctl->sm_rank[smid & 255u], 1u) % per_sm == 0u;
+        sm.red32[1][0] = leader;
+        sm.red32[1][1] = leader ? atomicAdd(&ctl->lead_cnt[lpar], 1u) : atomicAdd(&ctl->other_cnt[lpar], 1u);
+        if (blockIdx.x == 0) {
+            ctl->lead_cnt[lpar ^ 1u] = 0u;   // for the next launch (stream-ordered after this one)
+            ctl->other_cnt[lpar ^ 1u] = 0u;
+        }
+    }
     grid_barrier(ctl, a.nblocks);
+    const uint32_t nlead = ld_relaxed(&ctl->lead_cnt[lpar]);
+    const uint32_t vid = sm.red32[1][0] ? sm.red32[1][1] : nlead + sm.red32[1][1];   // permutation of [0, nblocks)
+    const uint32_t vgtid = vid * BS + threadIdx.x;
+    __syncthreads();   // (red32 reuse)
     uint32_t n = (ALG == ALG_CC) ? a.V : 1u;   // |WS_0| = |{src}| (CC: every vertex)
+    uint32_t nact = a.nblocks;   // CTAs taking part in the current iteration: vid < nact
+    const bool small_ok = TUNED && !a.has_hubs && a.pol.t_small > 0 && nlead > 0 && nlead < a.nblocks;
 
     uint32_t prev_ws = WS_QU;   // representation used in the previous iteration
     uint8_t prev_var = 0;
@@ -1010,19 +1033,57 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     uint32_t it = 0;
     bool in_raw = false;   // this iteration's working set is the raw bitmap of a free-output iteration
     for (;; ++it) {
-        const uint32_t slot = it % 3;
         if (TUNED && in_raw) {
-            compact_raw<ALG>(a, sm, a.bm[slot], it, a.q[slot], &ctl->q_len[slot]);
-            grid_barrier(ctl, a.nblocks);
-            n = ld_relaxed(&ctl->q_len[slot]);
+            compact_raw<ALG>(a, sm, a.bm[it % 3], it, a.q[it % 3], &ctl->q_len[it % 3], nact, vid);
+            grid_barrier(ctl, nact, vid == 0);
+            n = ld_relaxed(&ctl->q_len[it % 3]);
         }
         if (n == 0 || it >= a.max_iters) break;
+        if (small_ok) {
+            // small-frontier mode: below t_small only CTAs [0, small_ctas) run the iteration (the grid
+            // barrier then has small_ctas arrivals); the others park until CTA 0 wakes them with the
+            // iteration to resume at.  Every CTA takes the same decision (same n).
+            const uint32_t want = n < a.pol.t_small ? nlead : a.nblocks;
+            if (want > nact) {          // grow: wake the parked CTAs into this iteration
+                if (vid == 0 && threadIdx.x == 0) {
+                    ctl->wake_it = it;
+                    ctl->wake_n = n;
+                    ctl->wake_nprev = n_prev;
+                    __threadfence();
+                    st_release(&ctl->wake_gen, wgen + 1u);
+                }
+                wgen += 1u;
+                nact = want;
+            } else if (want < nact) {   // shrink
+                nact = want;
+                if (vid >= nact) {
+                    if (threadIdx.x == 0) {
+                        while (ld_relaxed(&ctl->wake_gen) == wgen) __nanosleep(1000);
+                        (void)ld_acquire(&ctl->wake_gen);
+                        sm.red32[1][0] = ld_relaxed(&ctl->wake_it);
+                        sm.red32[1][1] = ld_relaxed(&ctl->wake_n);
+                        sm.red32[1][2] = ld_relaxed(&ctl->wake_nprev);
+                    }
+                    __syncthreads();
+                    wgen += 1u;
+                    it = sm.red32[1][0];
+                    n = sm.red32[1][1];
+                    n_prev = sm.red32[1][2];
+                    __syncthreads();
+                    nact = a.nblocks;
+                    prev_var = 0;
+                    if (n == 0) break;      // the small group finished: join the final pass
+                }
+            }
+        }
+        const uint32_t slot = it % 3;
+        const uint32_t gact = nact * BS;   // threads taking part (grid-strided loops of this iteration)
         AG_PROF_MARK(it, 0);
         // decision maker, re-evaluated every sample_every iterations (inspector sampling, 26.s7-9)
         const uint8_t var = (it % a.pol.sample_every == 0 || prev_var == 0) ? select_variant(a.pol, n, 0) : prev_var;
         const uint32_t map = TUNED ? ((var >> 2) == MAP_T ? (uint32_t)MAP_T : (uint32_t)MAP_H) : (var >> 2);
         const uint32_t ws = TUNED ? (uint32_t)WS_QU : (var & 3u);
-        if (blockIdx.x == 0 && threadIdx.x == 0) {
+        if (vid == 0 && threadIdx.x == 0) {
             if (it < a.trace_cap && a.trace_ws) {
                 a.trace_ws[it] = n;
                 a.trace_var[it] = var;
@@ -1054,8 +1115,8 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             if (ws == WS_QU) {
                 if (prev_ws != WS_QU) {
                     // the pending list is stale: rebuild it from the pending bitmap
-                    compact_bitmap(a.bm[0], a.nwords, a.q[slot], &ctl->q_len[slot], gtid >> 5, gthreads >> 5);
-                    grid_barrier(ctl, a.nblocks);
+                    compact_bitmap(a.bm[0], a.nwords, a.q[slot], &ctl->q_len[slot], vgtid >> 5, gact >> 5);
+                    grid_barrier(ctl, nact, vid == 0);
                     qn = ld_relaxed(&ctl->q_len[slot]);
                 } else {
                     qn = ld_relaxed(&ctl->q_len[slot]);
@@ -1067,15 +1128,16 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             if (it > 0) {
                 if ((unsigned long long)n_prev * 32ull < a.nwords) {
                     const uint32_t *qp = a.q[(it + 2) % 3];
-                    for (uint32_t i = gtid; i < n_prev; i += gthreads) bz[qp[i] >> 5] = 0u;
+                    for (uint32_t i = vgtid; i < n_prev; i += gact) bz[qp[i] >> 5] = 0u;
                 } else {
-                    for (uint32_t wi = gtid; wi < a.nwords; wi += gthreads) bz[wi] = 0u;
+                    for (uint32_t wi = vgtid; wi < a.nwords; wi += gact) bz[wi] = 0u;
                 }
             }
         }
 
         Ops<ALG, ORD, Off> ops(a, it, hi, append);
         ops.wbuf = sm.wq[threadIdx.x >> 5];
+        ops.nact = nact;
         // free output (tuned, unordered, big working sets; BFS only without parents: a claim decides them)
         ops.freeo = TUNED && ROT && (ALG != ALG_BFS ? (uint64_t)qn >= a.pol.t_free_sssp
                                                     : ((uint64_t)qn >= a.pol.t_free && a.parent == nullptr));
@@ -1087,7 +1149,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         // mappings a short queue is spread over all CTAs (>= 2 tiles per CTA)
         uint32_t tile_n = BS;
         if (ws == WS_QU && map != MAP_T) {
-            uint32_t want = (qn + 2 * a.nblocks - 1) / (2 * a.nblocks);
+            uint32_t want = (qn + 2 * nact - 1) / (2 * nact);
             tile_n = want < 1u ? 1u : (want > (uint32_t)BS ? (uint32_t)BS : want);
         }
         // entry slot of this thread: spread across warps for the warp mapping
@@ -1099,10 +1161,11 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         {
             // dynamic tile scheduler: first tile static, then one atomic per tile, fetched one tile ahead
             // (double-buffered in smem; the __syncthreads_or below orders the write before the read)
-            uint32_t t = blockIdx.x;
+            uint32_t t = vid;
             int par = 0;
             while (t < ntiles) {
-                if (threadIdx.x == 0) sm.tnext[par] = a.nblocks + atomicAdd(&ctl->tile_ctr[slot], 1u);
+                // (no dynamic tiles when every tile is a static first tile: no atomic on the critical path)
+                if (threadIdx.x == 0) sm.tnext[par] = ntiles > nact ? nact + atomicAdd(&ctl->tile_ctr[slot], 1u) : ntiles;
                 bool valid;
                 uint32_t u;
                 if (ws == WS_BM) {
@@ -1124,7 +1187,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         AG_PROF_MARK(it, 2);
         ops.warp_flush(true);
         block_reduce_flush(ops, sm, ctl, slot);
-        grid_barrier(ctl, a.nblocks);
+        grid_barrier(ctl, nact, vid == 0);
         if (ops.freeo) {
             n = ld_relaxed(&ctl->free_any[(it + 1) % 3]) ? 1u : 0u;   // exact size after the compaction
             in_raw = true;
@@ -1138,7 +1201,14 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     }
 
     // ---------------- termination ----------------
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
+    if (nact < a.nblocks && vid == 0 && threadIdx.x == 0) {   // wake the parked CTAs for the final pass
+        ctl->wake_it = it;
+        ctl->wake_n = 0u;
+        ctl->wake_nprev = 0u;
+        __threadfence();
+        st_release(&ctl->wake_gen, wgen + 1u);
+    }
+    if (vid == 0 && threadIdx.x == 0) {
         ctl->iterations = it;
         if (it > 0 && it - 1 < a.trace_cap && a.trace_edges) a.trace_edges[it - 1] = ld_relaxed64(&ctl->it_edges[(it + 2) % 3]);
         if (it >= a.max_iters) ctl->aborted = 1;

@@ -323,3 +323,40 @@ def test_torch_allocator_hook():
         assert torch.cuda.memory_allocated() == before
     finally:
         A.use_torch_allocator(False)
+
+
+# ------------------------------------------------------------------------------------------------
+# small-frontier mode (tuned kernels on graphs without hub tasks): iterations with |WS| < t_small run
+# on one CTA per SM while the rest park; thresholds forced low so the group shrinks and grows many
+# times inside one traversal (env AG_SMALL_WS is read per query)
+# ------------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("t_small", ["1", "8", "100", "5000", "0"])
+def test_small_frontier_mode_transitions(t_small, monkeypatch):
+    monkeypatch.setenv("AG_SMALL_WS", t_small)
+    graphs = [aggen.config("C1"), aggen.with_weights(aggen.grid(60, 50), seed=9, wmax=100),
+              aggen.with_weights(aggen.er(5000, 20000, seed=4), seed=5, wmax=100),
+              aggen.random_graph(3000, 9000, seed=12)]
+    for g in graphs:
+        for layout in (1, 2):
+            G = A.Graph.from_csr(g, layout=layout)
+            lab = oracle.cc(g)
+            for s in sorted(set(int(x) for x in aggen.sources(g, 2)) | {0}):
+                check_bfs(g, G, s, pol(0), want_parents=False)
+                check_bfs(g, G, s, pol(0))
+                check_bfs(g, G, s, pol(1))
+                check_sssp(g, G, s, pol(0))
+                check_sssp(g, G, s, pol(0, free_ppm=1000000))
+                check_sssp(g, G, s, pol(1, delta=4))
+            assert np.array_equal(G.cc(policy=pol(0))[0], lab)
+            assert np.array_equal(G.cc(policy=pol(0, free_ppm=1000000))[0], lab)
+
+
+@pytest.mark.parametrize("cfg", ["C3", "C4"])
+def test_small_frontier_mode_full_size(cfg, monkeypatch):
+    """Default threshold on the latency-bound grid and on ER (frontier grows through t_small and back)."""
+    monkeypatch.delenv("AG_SMALL_WS", raising=False)
+    g = aggen.config(cfg)
+    G = A.Graph.from_csr(g)
+    for s in [int(x) for x in aggen.sources(g, 1)]:
+        check_bfs(g, G, s, pol(0), want_parents=False)
+        check_sssp(g, G, s, pol(0))
