@@ -135,12 +135,13 @@ struct Ops {
     bool ovf;
     bool freeo = false;     // free output: next working set = raw bitmap by fire-and-forget reductions
     bool any = false;       //   ... and this thread set at least one bit of it
-    uint32_t nact = 0;      // CTAs taking part in this iteration
+    uint32_t nact;          // CTAs taking part in this iteration (default: the whole grid)
+    bool bm_upd = true;     // BFS: write the update-vector bitmap (tuned queue-only kernels never read it)
 
     __device__ Ops(const TravArgs<Off> &a_, uint32_t it_, uint64_t hi_, bool append_)
         : a(a_), it(it_), hi(hi_), append_next(append_), fenced(ALG == ALG_SSSP && ORD == ORD_O && a_.pol.delta > 1),
           pol_stream(policy_evict_first()), pol_keep(policy_evict_last()), wbuf(nullptr), wfill(0), ne(0), nv(0),
-          vmin(INF), dpend(0), ovf(false) {
+          vmin(INF), dpend(0), ovf(false), nact(a_.nblocks) {
         const uint32_t sn = (it_ + 1) % 3;
         bm_next = (ALG == ALG_SSSP && ORD == ORD_O) ? a_.bm[0] : a_.bm[sn];
         q_next = a_.q[sn];
@@ -366,10 +367,10 @@ struct Ops {
                 if (won) {
                     if constexpr (ORD == ORD_O) {
                         a.level[v[j]] = nl;                            // m.level = level    (l.9)
-                        red_or(a.bm[(it + 1) % 3] + (v[j] >> 5), m);   // update vector      (l.10)
+                        if (bm_upd) red_or(a.bm[(it + 1) % 3] + (v[j] >> 5), m);   // update vector (l.10)
                     } else {
                         red_or(a.vis + (v[j] >> 5), m);
-                        red_or(bm_next + (v[j] >> 5), m);
+                        if (bm_upd) red_or(bm_next + (v[j] >> 5), m);
                     }
                     if (a.parent) a.parent[v[j]] = u[j];
                     nwm |= 1u << j;
@@ -1122,8 +1123,9 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
                     qn = ld_relaxed(&ctl->q_len[slot]);
                 }
             }
-        } else {
-            // clear the bitmap that iteration it+1 will write: bm[(it+2)%3] (read in iteration it-1)
+        } else if (!TUNED) {
+            // clear the bitmap that iteration it+1 will write: bm[(it+2)%3] (read in iteration it-1).
+            // (tuned kernels instead clear each frontier word when its vertex is read from the queue)
             uint32_t *bz = a.bm[(it + 2) % 3];
             if (it > 0) {
                 if ((unsigned long long)n_prev * 32ull < a.nwords) {
@@ -1138,6 +1140,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         Ops<ALG, ORD, Off> ops(a, it, hi, append);
         ops.wbuf = sm.wq[threadIdx.x >> 5];
         ops.nact = nact;
+        ops.bm_upd = !(TUNED && ALG == ALG_BFS);
         // free output (tuned, unordered, big working sets; BFS only without parents: a claim decides them)
         ops.freeo = TUNED && ROT && (ALG != ALG_BFS ? (uint64_t)qn >= a.pol.t_free_sssp
                                                     : ((uint64_t)qn >= a.pol.t_free && a.parent == nullptr));
@@ -1175,6 +1178,9 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
                     uint32_t i = t * tile_n + s_idx;
                     valid = s_idx < tile_n && i < qn;
                     u = valid ? qc[i] : 0u;
+                    // tuned, rotating bitmaps: every set bit of this iteration's bitmap is a queued vertex and
+                    // nothing reads the bitmap any more, so its words are cleared here for reuse in it+3
+                    if (TUNED && ROT && ALG != ALG_BFS && valid) a.bm[slot][u >> 5] = 0u;
                 }
                 if (__syncthreads_or(valid))  // skip empty tiles (sparse bitmap): uniform branch
                     process_tile<TUNED>(ops, sm, map, valid, u, a.pol.cta_group, hubs, slot);
