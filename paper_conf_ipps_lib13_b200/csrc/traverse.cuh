@@ -151,6 +151,9 @@ struct Ops {
     // Is working-set element u expanded in this iteration?  Fills its adjacency range and value.
     __device__ __forceinline__ bool gate(uint32_t u, Off &beg, uint32_t &deg, uint32_t &uval) {
         bool ex = true;
+        // the adjacency range is loaded first, in parallel with the value that decides (SSSP): nearly
+        // every working-set element is expanded, and the two loads no longer wait for each other
+        const Off rb = a.rp[u], re = a.rp[u + 1];
         if constexpr (ALG == ALG_BFS) {
             uval = it;  // the frontier of iteration it is exactly level it (level-synchronous, 26.s33)
         } else if constexpr (ALG == ALG_CC) {
@@ -180,7 +183,7 @@ struct Ops {
                     vmin = min(vmin, t);
                 }
                 if (append_next) warp_append(q_next, qlen_next, !ex && (uint64_t)t >= hi, u);
-            } else if ((uint64_t)t >= hi || ((uint64_t)t >= hub_hi && (uint32_t)(a.rp[u + 1] - a.rp[u]) >= HUBW_DEG)) {
+            } else if ((uint64_t)t >= hi || ((uint64_t)t >= hub_hi && (uint32_t)(re - rb) >= HUBW_DEG)) {
                 // unordered SSSP with a deferral window: a far vertex stays in the working set
                 // (re-added to the next frontier unless an improvement already did) and feeds the
                 // minimum that places the next window
@@ -197,9 +200,8 @@ struct Ops {
             }
         }
         if (ex) {
-            beg = a.rp[u];
-            Off end = a.rp[u + 1];
-            deg = (uint32_t)(end - beg);
+            beg = rb;
+            deg = (uint32_t)(re - rb);
             nv += 1;
             ne += deg;
         } else {
