@@ -9,6 +9,10 @@
 #include <cstring>
 #include <mutex>
 #include <string>
+#include <vector>
+
+#include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_scan.cuh>
 
 #include "agraph.h"
 #include "common.cuh"
@@ -166,6 +170,41 @@ __global__ void validate_edges_kernel(const uint32_t *col, const uint32_t *w, ui
             uint32_t x = w[e];
             if (x == 0 || x >= 0x80000000u) bad |= 16;
             mw = max(mw, x);
+        }
+    }
+    bad = __reduce_or_sync(0xffffffffu, bad);
+    mw = __reduce_max_sync(0xffffffffu, mw);
+    if ((threadIdx.x & 31) == 0) {
+        if (bad) atomicOr(&st->bad, bad);
+        if (mw) atomicMax(&st->max_w, mw);
+    }
+}
+
+// Degree layout, one chunk of the pipelined load: the CSR entries of old rows [ra, rb) (all arrived) go to
+// their relabelled positions nrp[inv[u]] + (e - rp[u]) with the neighbour mapped through inv (an
+// out-of-range id is flagged, never dereferenced); weights are validated and interleaved into cw.
+// Edge-parallel (one owner binary search per entry) so hub rows do not serialise on one warp.
+__global__ void relabel_edges_kernel(const uint64_t *rp, const uint32_t *col, const uint32_t *w, const uint32_t *inv,
+                                     const uint64_t *nrp, uint32_t V, uint32_t ra, uint32_t rb, uint32_t *ncol, uint2 *cw,
+                                     LoadStats *st) {
+    const uint64_t e0 = rp[ra], e1 = rp[rb];
+    unsigned bad = 0, mw = 0;
+    for (uint64_t e = e0 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < e1; e += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t lo = ra, hi = rb;   // rp[lo] <= e < rp[hi]: the owner is the largest u with rp[u] <= e
+        while (hi - lo > 1) {
+            const uint32_t mid = lo + (hi - lo) / 2;
+            if (rp[mid] <= e) lo = mid; else hi = mid;
+        }
+        const uint32_t c = col[e];
+        uint32_t nc = 0;
+        if (c < V) nc = inv[c]; else bad |= 8;
+        const uint64_t ne = nrp[inv[lo]] + (e - rp[lo]);
+        ncol[ne] = nc;
+        if (w) {
+            const uint32_t x = w[e];
+            if (x == 0 || x >= 0x80000000u) bad |= 16;
+            mw = max(mw, x);
+            cw[ne] = make_uint2(nc, x);
         }
     }
     bad = __reduce_or_sync(0xffffffffu, bad);
@@ -665,72 +704,164 @@ ag_status ag_graph_load_csr_ex(uint32_t V, uint64_t E, const uint64_t *row_ptr, 
     cudaEventCreate(&g->ev[1]);
     auto fail = [&](ag_status st) { ag_graph_free(g); return st; };
 
+    // ---- pipelined load (row a1): the row offsets are copied and validated first
+    // (the inspector's degree statistics decide the layout), then col_idx / weights stream in
+    // CH-edge chunks on a copy stream while a processing stream validates each chunk and builds the
+    // final arrays from it (identity: the (col, w) interleave; degree layout: the relabelled rows
+    // whose last entry is in the chunk).  The host waits once, so the PCIe copy hides the processing.
+    LoadStats hs = {0, 0xFFFFFFFFu, 0, 0, 0};
     uint64_t *rp64 = nullptr;
     LoadStats *dst = nullptr;
-    if ((s = dev_alloc((void **)&rp64, (size_t)(V + 1) * 8, device)) != AG_OK) return fail(s);
-    if ((s = dev_alloc((void **)&g->d_col, E * 4 + 128, device)) != AG_OK) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(s); }
-    g->col_bytes = E * 4 + 128;
-    if (weights) {
-        if ((s = dev_alloc((void **)&g->d_w, E * 4 + 128, device)) != AG_OK) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(s); }
-        g->w_bytes = E * 4 + 128;
-    }
-    if ((s = dev_alloc((void **)&dst, sizeof(LoadStats), device)) != AG_OK) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(s); }
-    cudaError_t e = cudaMemcpy(rp64, row_ptr, (size_t)(V + 1) * 8, cudaMemcpyDefault);
-    if (e == cudaSuccess && E) e = cudaMemcpy(g->d_col, col_idx, E * 4, cudaMemcpyDefault);
-    if (e == cudaSuccess && E && weights) e = cudaMemcpy(g->d_w, weights, E * 4, cudaMemcpyDefault);
-    LoadStats hs = {0, 0xFFFFFFFFu, 0, 0, 0};
-    if (e == cudaSuccess) e = cudaMemcpy(dst, &hs, sizeof hs, cudaMemcpyHostToDevice);
+    uint32_t *col_old = nullptr, *w_old = nullptr;   // staging (freed at the end of the load)
+    unsigned long long *keys = nullptr, *keys2 = nullptr;
+    uint64_t *ndeg = nullptr, *nrp = nullptr;
+    void *tmp = nullptr;
+    size_t tmp_bytes = 0;
+    uint64_t *rp_host = nullptr;   // host copy of row_ptr when the caller passed device memory (degree layout)
+    cudaStream_t s_copy = nullptr, s_proc = nullptr;
+    std::vector<cudaEvent_t> evs;
+    auto release = [&]() {
+        if (s_copy) cudaStreamSynchronize(s_copy);
+        if (s_proc) cudaStreamSynchronize(s_proc);
+        for (auto ev : evs) cudaEventDestroy(ev);
+        evs.clear();
+        if (s_copy) cudaStreamDestroy(s_copy);
+        if (s_proc) cudaStreamDestroy(s_proc);
+        s_copy = s_proc = nullptr;
+        dev_free(rp64, (size_t)(V + 1) * 8 + 8, device);
+        dev_free(dst, sizeof(LoadStats), device);
+        dev_free(col_old, E * 4 + 128, device);
+        dev_free(w_old, E * 4 + 128, device);
+        dev_free(keys, (size_t)V * 8, device);
+        dev_free(keys2, (size_t)V * 8, device);
+        dev_free(ndeg, (size_t)V * 8 + 8, device);
+        dev_free(nrp, (size_t)V * 8 + 8, device);
+        dev_free(tmp, tmp_bytes, device);
+        free(rp_host);
+        rp64 = nullptr; dst = nullptr; col_old = w_old = nullptr; keys = keys2 = nullptr; ndeg = nrp = nullptr;
+        tmp = nullptr; rp_host = nullptr;
+    };
+    auto lfail = [&](ag_status st) { release(); return fail(st); };
+    cudaError_t e = cudaStreamCreateWithFlags(&s_copy, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&s_proc, cudaStreamNonBlocking);
+    if (e != cudaSuccess) return lfail(cuda_status(e, "load streams"));
+    if ((s = dev_alloc((void **)&rp64, (size_t)(V + 1) * 8 + 8, device)) != AG_OK) return lfail(s);
+    if ((s = dev_alloc((void **)&dst, sizeof(LoadStats), device)) != AG_OK) return lfail(s);
+    e = cudaMemcpyAsync(rp64, row_ptr, (size_t)(V + 1) * 8, cudaMemcpyDefault, s_proc);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(dst, &hs, sizeof hs, cudaMemcpyHostToDevice, s_proc);
     if (e == cudaSuccess) {
-        validate_rows_kernel<<<sms * 8, 256>>>(rp64, V, E, dst);
-        if (E) validate_edges_kernel<<<sms * 8, 256>>>(g->d_col, weights ? g->d_w : nullptr, E, V, dst);
-        note_launch(E ? 2 : 1);
-        e = cudaMemcpy(&hs, dst, sizeof hs, cudaMemcpyDeviceToHost);
+        validate_rows_kernel<<<sms * 8, 256, 0, s_proc>>>(rp64, V, E, dst);
+        note_launch(1);
+        e = cudaMemcpyAsync(&hs, dst, sizeof hs, cudaMemcpyDeviceToHost, s_proc);
     }
-    dev_free(dst, sizeof(LoadStats), device);
-    if (e != cudaSuccess) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(cuda_status(e, "graph load")); }
-    if (hs.bad) {
-        dev_free(rp64, (size_t)(V + 1) * 8, device);
-        return fail(set_error(AG_ERR_BAD_CSR, "invalid CSR (%s%s%s%s%s)", hs.bad & 1 ? "row_ptr[0]!=0 " : "",
-                              hs.bad & 2 ? "non-monotone row_ptr " : "", hs.bad & 4 ? "row_ptr[V]!=E " : "",
-                              hs.bad & 8 ? "col>=V " : "", hs.bad & 16 ? "weight not in [1,2^31) " : ""));
-    }
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s_proc);
+    if (e != cudaSuccess) return lfail(cuda_status(e, "graph load"));
+    if (hs.bad)
+        return lfail(set_error(AG_ERR_BAD_CSR, "invalid CSR (%s%s%s)", hs.bad & 1 ? "row_ptr[0]!=0 " : "",
+                               hs.bad & 2 ? "non-monotone row_ptr " : "", hs.bad & 4 ? "row_ptr[V]!=E " : ""));
     // inspector decides the device layout (skewed degree distribution -> degree order)
     if (layout == AG_LAYOUT_AUTO) {
         uint64_t avg = (E + V - 1) / V;
         layout = (E > 0 && (uint64_t)hs.max_deg >= 64ull * (avg ? avg : 1)) ? AG_LAYOUT_DEGREE : AG_LAYOUT_IDENTITY;
     }
     g->layout = layout;
-    if (layout == AG_LAYOUT_DEGREE) {
-        uint64_t *nrp = nullptr;
-        if ((s = build_degree_layout(g, rp64, &nrp)) != AG_OK) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(s); }
-        dev_free(rp64, (size_t)(V + 1) * 8, device);
-        rp64 = nrp;  // (allocated with V*8+8 bytes)
+    const bool deg = layout == AG_LAYOUT_DEGREE;
+    // final arrays
+    if ((s = dev_alloc((void **)&g->d_col, E * 4 + 128, device)) != AG_OK) return lfail(s);
+    g->col_bytes = E * 4 + 128;
+    if (weights) {
+        if ((s = dev_alloc((void **)&g->d_cw, E * 8 + 128, device)) != AG_OK) return lfail(s);
+        g->cw_bytes = E * 8 + 128;
+        if ((s = dev_alloc((void **)&w_old, E * 4 + 128, device)) != AG_OK) return lfail(s);
     }
+    if (deg) {
+        if ((s = dev_alloc((void **)&col_old, E * 4 + 128, device)) != AG_OK) return lfail(s);
+        if ((s = dev_alloc((void **)&keys, (size_t)V * 8, device)) != AG_OK) return lfail(s);
+        if ((s = dev_alloc((void **)&keys2, (size_t)V * 8, device)) != AG_OK) return lfail(s);
+        if ((s = dev_alloc((void **)&ndeg, (size_t)V * 8 + 8, device)) != AG_OK) return lfail(s);
+        if ((s = dev_alloc((void **)&nrp, (size_t)V * 8 + 8, device)) != AG_OK) return lfail(s);
+        if ((s = dev_alloc((void **)&g->d_perm, (size_t)V * 4, device)) != AG_OK) return lfail(s);
+        if ((s = dev_alloc((void **)&g->d_inv, (size_t)V * 4, device)) != AG_OK) return lfail(s);
+        size_t t1 = 0, t2 = 0;
+        cub::DeviceRadixSort::SortKeys(nullptr, t1, keys, keys2, (int)V);
+        cub::DeviceScan::ExclusiveSum(nullptr, t2, ndeg, nrp, (int)V + 1);
+        tmp_bytes = t1 > t2 ? t1 : t2;
+        if ((s = dev_alloc(&tmp, tmp_bytes, device)) != AG_OK) return lfail(s);
+        if (is_device_ptr(row_ptr)) {   // the chunk -> row ranges are found on the host
+            rp_host = (uint64_t *)malloc((size_t)(V + 1) * 8);
+            if (!rp_host) return lfail(set_error(AG_ERR_OOM, "host row_ptr copy"));
+            e = cudaMemcpy(rp_host, row_ptr, (size_t)(V + 1) * 8, cudaMemcpyDeviceToHost);
+            if (e != cudaSuccess) return lfail(cuda_status(e, "row_ptr readback"));
+        }
+        // degree order and new row offsets (overlaps the edge copies below)
+        build_degree_order(rp64, V, keys, keys2, tmp, tmp_bytes, g->d_perm, g->d_inv, ndeg, nrp, sms, s_proc);
+    }
+    const uint64_t *rph = rp_host ? rp_host : row_ptr;
+    uint32_t *col_dst = deg ? col_old : g->d_col;
+    const uint64_t CH = 1ull << 24;   // edges per chunk (64 MB of col_idx, 64 MB of weights)
+    uint32_t row_a = 0;
+    for (uint64_t e0 = 0; e0 < E; e0 += CH) {
+        const uint64_t e1 = (E - e0 > CH) ? e0 + CH : E;
+        cudaEvent_t ev;
+        if ((e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) != cudaSuccess) return lfail(cuda_status(e, "event"));
+        evs.push_back(ev);
+        e = cudaMemcpyAsync(col_dst + e0, col_idx + e0, (e1 - e0) * 4, cudaMemcpyDefault, s_copy);
+        if (e == cudaSuccess && weights) e = cudaMemcpyAsync(w_old + e0, weights + e0, (e1 - e0) * 4, cudaMemcpyDefault, s_copy);
+        if (e == cudaSuccess) e = cudaEventRecord(ev, s_copy);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(s_proc, ev, 0);
+        if (e != cudaSuccess) return lfail(cuda_status(e, "edge copy"));
+        const int grid = sms * 8;
+        if (!deg) {
+            validate_edges_kernel<<<grid, 256, 0, s_proc>>>(g->d_col + e0, weights ? w_old + e0 : nullptr, e1 - e0, V, dst);
+            if (weights) interleave_kernel<<<grid, 256, 0, s_proc>>>(g->d_col + e0, w_old + e0, g->d_cw + e0, e1 - e0);
+            note_launch(weights ? 2 : 1);
+        } else {
+            // rows whose last entry lies in [e0, e1) (all their entries have arrived): rp[u+1] <= e1
+            uint32_t lo = row_a, hi = V;   // first u in [row_a, V] with rp[u+1] > e1 (V if none)
+            if (e1 < E) {
+                while (lo < hi) {
+                    const uint32_t mid = lo + (hi - lo) / 2;
+                    if (rph[mid + 1] > e1) hi = mid; else lo = mid + 1;
+                }
+            } else {
+                lo = V;
+            }
+            if (lo > row_a) {
+                relabel_edges_kernel<<<grid, 256, 0, s_proc>>>(rp64, col_old, weights ? w_old : nullptr, g->d_inv, nrp, V,
+                                                               row_a, lo, g->d_col, g->d_cw, dst);
+                note_launch(1);
+            }
+            row_a = lo;
+        }
+    }
+    // final row offsets (u32 when E < 2^32)
+    const uint64_t *rp_final = deg ? nrp : rp64;
     if (g->offs32) {
         uint32_t *rp32 = nullptr;
-        if ((s = dev_alloc((void **)&rp32, (size_t)(V + 1) * 4 + 128, device)) != AG_OK) { dev_free(rp64, (size_t)(V + 1) * 8, device); return fail(s); }
-        narrow_offsets_kernel<<<sms * 8, 256>>>(rp64, rp32, V + 1);
-        note_launch(1);
-        e = cudaDeviceSynchronize();
-        dev_free(rp64, (size_t)(V + 1) * 8, device);
-        if (e != cudaSuccess) { dev_free(rp32, (size_t)(V + 1) * 4 + 128, device); return fail(cuda_status(e, "narrow")); }
+        if ((s = dev_alloc((void **)&rp32, (size_t)(V + 1) * 4 + 128, device)) != AG_OK) return lfail(s);
         g->d_rp = rp32;
         g->rp_bytes = (size_t)(V + 1) * 4 + 128;
-    } else {
-        g->d_rp = rp64;
-        g->rp_bytes = (size_t)(V + 1) * 8;
-    }
-    if (g->d_w) {  // SSSP reads (col, w) together: interleave, drop the separate weight array
-        if ((s = dev_alloc((void **)&g->d_cw, E * 8 + 128, device)) != AG_OK) return fail(s);
-        g->cw_bytes = E * 8 + 128;
-        if (E) interleave_kernel<<<sms * 8, 256>>>(g->d_col, g->d_w, g->d_cw, E);
+        narrow_offsets_kernel<<<sms * 8, 256, 0, s_proc>>>(rp_final, rp32, V + 1);
         note_launch(1);
-        e = cudaDeviceSynchronize();
-        if (e != cudaSuccess) return fail(cuda_status(e, "interleave"));
-        dev_free(g->d_w, g->w_bytes, device);
-        g->d_w = nullptr;
-        g->w_bytes = 0;
+    } else {
+        uint64_t *rpk = nullptr;
+        if ((s = dev_alloc((void **)&rpk, (size_t)(V + 1) * 8 + 8, device)) != AG_OK) return lfail(s);
+        g->d_rp = rpk;
+        g->rp_bytes = (size_t)(V + 1) * 8 + 8;
+        e = cudaMemcpyAsync(rpk, rp_final, (size_t)(V + 1) * 8, cudaMemcpyDeviceToDevice, s_proc);
+        if (e != cudaSuccess) return lfail(cuda_status(e, "row offsets"));
     }
+    LoadStats he = hs;
+    e = cudaMemcpyAsync(&he, dst, sizeof he, cudaMemcpyDeviceToHost, s_proc);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s_proc);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s_copy);
+    if (e == cudaSuccess) e = cudaGetLastError();
+    if (e != cudaSuccess) return lfail(cuda_status(e, "graph load"));
+    if (he.bad)
+        return lfail(set_error(AG_ERR_BAD_CSR, "invalid CSR (%s%s)", he.bad & 8 ? "col>=V " : "",
+                               he.bad & 16 ? "weight not in [1,2^31) " : ""));
+    hs.max_w = he.max_w;
+    release();
     g->info.num_vertices = V;
     g->info.num_edges = E;
     g->info.deg_sum = E;
