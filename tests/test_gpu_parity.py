@@ -360,3 +360,65 @@ def test_small_frontier_mode_full_size(cfg, monkeypatch):
     for s in [int(x) for x in aggen.sources(g, 1)]:
         check_bfs(g, G, s, pol(0), want_parents=False)
         check_sssp(g, G, s, pol(0))
+
+
+# ------------------------------------------------------------------------------------------------
+# pipelined graph load: several 16M-edge chunks, host and device inputs, both layouts, rows that span
+# chunk boundaries (hubs), and CSR errors found in a LATER chunk (after earlier chunks were processed)
+# ------------------------------------------------------------------------------------------------
+def test_pipelined_load_multichunk_host_and_device():
+    import torch
+    g = aggen.with_weights(aggen.rmat(20, 20, seed=7), seed=8, wmax=100)   # E ~ 38M: 3 chunks, hub rows span them
+    assert g.E > 2 * (1 << 24)
+    s = int(aggen.sources(g, 1, seed=5)[0])
+    lv, _ = oracle.bfs(g, s, want_parents=False)
+    d, _ = oracle.dijkstra(g, s, want_parents=False)
+    lab = oracle.cc(g)
+    t_rp = torch.from_numpy(g.row_ptr.view(np.int64)).cuda()
+    t_col = torch.from_numpy(g.col.view(np.int32)).cuda()
+    t_w = torch.from_numpy(g.w.view(np.int32)).cuda()
+    for layout in (1, 2):
+        for dev in (False, True):
+            G = A.Graph(g.V, t_rp, t_col, t_w, layout=layout) if dev else A.Graph.from_csr(g, layout=layout)
+            assert G.info.layout == layout and G.info.max_weight == int(g.w.max())
+            assert G.info.max_deg == int(np.diff(g.row_ptr).max())
+            assert np.array_equal(G.bfs(s)[0], lv)
+            assert np.array_equal(G.sssp(s)[0], d)
+            assert np.array_equal(G.cc()[0], lab)
+            G.free()
+
+
+@pytest.mark.parametrize("where", ["first", "last"])
+@pytest.mark.parametrize("layout", [1, 2])
+def test_pipelined_load_errors_in_any_chunk(where, layout):
+    g = aggen.with_weights(aggen.rmat(20, 20, seed=7), seed=8, wmax=100)
+    pos = 5 if where == "first" else g.E - 3
+    col = g.col.copy()
+    col[pos] = g.V                  # out-of-range neighbour
+    with pytest.raises(A.AgError) as e:
+        A.Graph(g.V, g.row_ptr, col, g.w, layout=layout)
+    assert e.value.status == "AG_ERR_BAD_CSR"
+    w = g.w.copy()
+    w[pos] = 0                      # zero weight
+    with pytest.raises(A.AgError) as e:
+        A.Graph(g.V, g.row_ptr, g.col, w, layout=layout)
+    assert e.value.status == "AG_ERR_BAD_CSR"
+    # the library is still usable after rejected loads
+    G = A.Graph.from_csr(g, layout=layout)
+    s = int(aggen.sources(g, 1, seed=5)[0])
+    assert np.array_equal(G.bfs(s)[0], oracle.bfs(g, s, want_parents=False)[0])
+
+
+def test_pipelined_load_degree_layout_edge_cases():
+    """Forced degree layout with no edges, with trailing isolated vertices, and unweighted."""
+    g0 = aggen.csr_from_edges(70, [], [], w=[])
+    G = A.Graph.from_csr(g0, layout=2)
+    assert list(G.bfs(3)[0]) == [INF] * 3 + [0] + [INF] * 66
+    assert np.array_equal(G.cc()[0], np.arange(70, dtype=np.uint32))
+    g = aggen.csr_from_edges(100, [0, 0, 1, 5], [1, 5, 2, 0], w=[3, 4, 5, 6])   # 6..99 isolated
+    for weighted in (True, False):
+        G = A.Graph.from_csr(g, layout=2, weighted=weighted)
+        assert np.array_equal(G.bfs(0)[0], oracle.bfs(g, 0)[0])
+        if weighted:
+            assert np.array_equal(G.sssp(0)[0], oracle.dijkstra(g, 0)[0])
+        assert np.array_equal(G.cc()[0], oracle.cc(g))
