@@ -37,7 +37,7 @@ namespace ag {
 // diagnostic build only: per (iteration, CTA) timestamps — iteration start, tile loop done, hub drain
 // done — read back with ag_debug_prof() (tools/prof_iters.py)
 constexpr int PROF_IT = 64, PROF_CTA = 2048;
-__device__ unsigned long long g_prof[PROF_IT][PROF_CTA][3];
+__device__ unsigned long long g_prof[PROF_IT][PROF_CTA][4];   // [3]: adjacency entries gated by the CTA's tiles
 #define AG_PROF_MARK(it, k) \
     if (threadIdx.x == 0 && (it) < PROF_IT && blockIdx.x < PROF_CTA) g_prof[it][blockIdx.x][k] = globaltimer_ns()
 #else
@@ -158,6 +158,14 @@ struct Ops {
             uval = it;  // the frontier of iteration it is exactly level it (level-synchronous, 26.s33)
         } else if constexpr (ALG == ALG_CC) {
             uval = ld_relaxed(&a.level[u]);   // the current label (never above the one that queued u)
+            // shortcut (pointer jumping): the label of u's label also reaches u, so u can take it before
+            // it is expanded — on a high-diameter graph the reach of a label doubles per iteration
+            // instead of growing by one hop (R23; results unchanged: same fixed point)
+            const uint32_t l2 = ld_relaxed(&a.level[a.inv ? a.inv[uval] : uval]);
+            if (l2 < uval) {
+                red_min32(&a.level[u], l2);
+                uval = l2;
+            }
         } else if (a.ulist) {
             // listed entry: uval (the sender's distance of u) was set by the caller; every entry expands
         } else {
@@ -1191,6 +1199,20 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             }
         }
         AG_PROF_MARK(it, 1);
+#ifdef AG_PROF
+        {
+            const unsigned long long x = warp_sum(ops.ne);
+            __syncthreads();
+            if (lane_id() == 0) sm.red64[0][threadIdx.x >> 5] = x;
+            __syncthreads();
+            if (threadIdx.x == 0 && it < PROF_IT && blockIdx.x < PROF_CTA) {
+                unsigned long long t = 0;
+                for (int w = 0; w < WARPS_PER_CTA; ++w) t += sm.red64[0][w];
+                g_prof[it][blockIdx.x][3] = t;
+            }
+            __syncthreads();
+        }
+#endif
         if (hubs) drain_hubs(ops, sm, slot);   // (begins with __syncthreads)
         AG_PROF_MARK(it, 2);
         ops.warp_flush(true);
