@@ -10,7 +10,7 @@ for cfg in ${AB_CONFIGS:-C2 C4}; do
   for alg in ${AB_ALGS:-bfs sssp}; do
     for L in exp_libs/*.so; do
       echo "== $cfg $alg $L"
-      AGRAPH_LIB=$PWD/$L timeout 300 python tools/one_query.py --config $cfg --alg $alg --n ${AB_N:-6} 2>&1 | tail -4
+      AGRAPH_LIB=$PWD/$L timeout 300 python tools/one_query.py --config $cfg --alg $alg --n ${AB_N:-6} --summary 2>&1 | tail -2
     done
   done
 done
