@@ -358,6 +358,8 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
     d.small_ctas = (uint32_t)g.num_sms;
     d.t_small = p.kind == AG_POLICY_TUNED ? 32768u : 0u;
     if (const char *ts = getenv("AG_SMALL_WS")) d.t_small = (uint32_t)atoi(ts);   // experiments / tests
+    d.t_small_hub = p.kind == AG_POLICY_TUNED ? 4096u : 0u;   // C2: BFS -1.6%, SSSP -2.7% (median of 12)
+    if (const char *ts = getenv("AG_SMALL_HUB_WS")) d.t_small_hub = (uint32_t)atoi(ts);
     return d;
 }
 

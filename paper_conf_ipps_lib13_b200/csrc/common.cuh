@@ -133,6 +133,7 @@ struct DevPolicy {
     uint64_t t_free_sssp; //   ... SSSP (never on skewed graphs: red.min on hot targets loses, tools/gpu_free_ab.sh)
     uint32_t small_ctas;  // tuned kernels: CTAs that run an iteration whose |WS| < t_small (the rest park)
     uint32_t t_small;     //   0 = off
+    uint32_t t_small_hub; //   graphs with hub tasks: only in the shrinking tail (|WS| below this and falling)
 };
 
 // The decision maker.  PAPER: Fig. 11 with readings R12/R13:

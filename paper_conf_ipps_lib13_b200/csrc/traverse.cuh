@@ -1036,7 +1036,8 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     __syncthreads();   // (red32 reuse)
     uint32_t n = (ALG == ALG_CC) ? a.V : 1u;   // |WS_0| = |{src}| (CC: every vertex)
     uint32_t nact = a.nblocks;   // CTAs taking part in the current iteration: vid < nact
-    const bool small_ok = TUNED && !a.has_hubs && a.pol.t_small > 0 && nlead > 0 && nlead < a.nblocks;
+    const bool small_ok = TUNED && (a.has_hubs ? a.pol.t_small_hub > 0 : a.pol.t_small > 0) && nlead > 0 &&
+                          nlead < a.nblocks;
 
     uint32_t prev_ws = WS_QU;   // representation used in the previous iteration
     uint8_t prev_var = 0;
@@ -1054,7 +1055,9 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             // small-frontier mode: below t_small only CTAs [0, small_ctas) run the iteration (the grid
             // barrier then has small_ctas arrivals); the others park until CTA 0 wakes them with the
             // iteration to resume at.  Every CTA takes the same decision (same n).
-            const uint32_t want = n < a.pol.t_small ? nlead : a.nblocks;
+            // (graphs with hub tasks: only in the falling tail, where the hubs have long been expanded)
+            const bool small = a.has_hubs ? (n < a.pol.t_small_hub && it > 0 && n < n_prev) : n < a.pol.t_small;
+            const uint32_t want = small ? nlead : a.nblocks;
             if (want > nact) {          // grow: wake the parked CTAs into this iteration
                 if (vid == 0 && threadIdx.x == 0) {
                     ctl->wake_it = it;
