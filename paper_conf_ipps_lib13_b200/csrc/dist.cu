@@ -97,9 +97,12 @@ struct ag_dist_part {
     // SSSP exchange buffers (allocated on the first ag_dist_sssp)
     uint2 *d_send = nullptr;           // S entries: (owned improved vertex, its distance)
     uint2 *d_list = nullptr;           // world * S entries: the gathered global frontier
-    unsigned *d_counts = nullptr;      // world per-rank counts (gathered)
+    unsigned *d_counts = nullptr;      // world x CW words per rank: (sent, carried, min pending dist, 0), gathered
     unsigned *h_counts = nullptr;      // pinned copy
+    uint32_t *d_carry[2] = {nullptr, nullptr};   // owned pending vertices held back (hub window), double-buffered
+    uint32_t *d_indeg = nullptr;       // in-degree of every owned vertex (all its in-edges live on this rank)
 };
+constexpr int CW = 4;                  // words per rank in the SSSP count exchange
 
 namespace ag {
 
@@ -113,8 +116,11 @@ void dist_graph_release(ag_graph_s *g) {
     const int W = d->comm ? d->comm->world : 1;
     dev_free(d->d_send, (size_t)d->S * 8 + 128, g->device);
     dev_free(d->d_list, (size_t)W * d->S * 8 + 128, g->device);
-    dev_free(d->d_counts, (size_t)W * 4 + 128, g->device);
+    dev_free(d->d_counts, (size_t)W * CW * 4 + 128, g->device);
     if (d->h_counts) cudaFreeHost(d->h_counts);
+    dev_free(d->d_carry[0], (size_t)d->S * 4 + 128, g->device);
+    dev_free(d->d_carry[1], (size_t)d->S * 4 + 128, g->device);
+    dev_free(d->d_indeg, (size_t)d->S * 4 + 128, g->device);
     delete d;
     g->dist = nullptr;
 }
@@ -266,18 +272,56 @@ __global__ void __launch_bounds__(BS, AG_MINB_SSSP) dist_sssp_kernel(const TravA
     block_reduce_flush(ops, sm, ctl, slot);
 }
 
-// The rank's contribution to the next global frontier: (v, dist v) for every owned v improved in this
-// round (the local next queue, deduplicated by the bitmap), read after the round so the latest
-// distance is sent; clears the next-bitmap words for the following round.
-__global__ void dist_sssp_collect_kernel(const uint32_t *q, const unsigned *qlen, const unsigned long long *P,
-                                         uint32_t *next_bm, uint2 *send, unsigned *count) {
-    const uint32_t n = *qlen;
-    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-        const uint32_t v = q[i];
-        send[i] = make_uint2(v, (uint32_t)(P[v] >> 32));
-        next_bm[v >> 5] = 0u;
+// The rank's contribution to the next global frontier, decided by the OWNER (so every rank expands the
+// same list): its pending vertices are the ones held back last round (cin) and the ones improved in this
+// round (q, deduplicated by the pending bitmap).  A pending vertex is sent as (v, dist v) — its latest
+// distance — unless it is a hub (in-degree >= HUBW_DEG: re-expanding it re-scans its whole list on every
+// rank) whose distance is at least `hi` = (global minimum pending distance of the last exchange) +
+// hub window; those stay pending (cout, bit kept set).  Sent vertices leave the pending bitmap.
+// cnt[0] = sent, cnt[1] = carried, cnt[2] = minimum pending distance (all zeroed / INF by the caller).
+// The hub window only reorders work: the global minimum pending vertex is always sent next round.
+__global__ void dist_sssp_collect_kernel(const uint32_t *cin, uint32_t ncin, const uint32_t *q, const unsigned *qlen,
+                                         const unsigned long long *P, const uint32_t *indeg, uint32_t own_b,
+                                         unsigned long long hi, uint32_t *pend_bm, uint2 *send, uint32_t *cout,
+                                         unsigned *cnt) {
+    const uint32_t nq = *qlen, tot = ncin + nq;
+    uint32_t lmin = INF;
+    const uint32_t gs = gridDim.x * blockDim.x;
+    for (uint32_t i0 = blockIdx.x * blockDim.x; i0 < tot; i0 += gs) {   // warp-uniform trip count
+        const uint32_t i = i0 + threadIdx.x;
+        bool ok = i < tot, snd = false;
+        uint32_t v = 0, dv = INF;
+        if (ok) {
+            v = i < ncin ? cin[i] : q[i - ncin];
+            dv = (uint32_t)(P[v] >> 32);
+            lmin = min(lmin, dv);
+            snd = indeg[v - own_b] < HUBW_DEG || (unsigned long long)dv < hi;
+        }
+        const unsigned ms = __ballot_sync(0xffffffffu, ok && snd), mc = __ballot_sync(0xffffffffu, ok && !snd);
+        const unsigned lane = threadIdx.x & 31u, below = (1u << lane) - 1u;
+        uint32_t bs = 0, bc = 0;
+        if (lane == 0) {
+            if (ms) bs = atomicAdd(&cnt[0], (unsigned)__popc(ms));
+            if (mc) bc = atomicAdd(&cnt[1], (unsigned)__popc(mc));
+        }
+        bs = __shfl_sync(0xffffffffu, bs, 0);
+        bc = __shfl_sync(0xffffffffu, bc, 0);
+        if (ok && snd) {
+            send[bs + __popc(ms & below)] = make_uint2(v, dv);
+            atomicAnd(&pend_bm[v >> 5], ~(1u << (v & 31)));
+        } else if (ok) {
+            cout[bc + __popc(mc & below)] = v;
+        }
     }
-    if (blockIdx.x == 0 && threadIdx.x == 0) *count = n;
+    lmin = warp_min(lmin);
+    if ((threadIdx.x & 31u) == 0 && lmin != INF) atomicMin(&cnt[2], lmin);
+}
+
+// in-degree of the owned vertices: every CSR entry of this rank has an owned destination
+__global__ void dist_indeg_kernel(const uint32_t *col, unsigned long long E, uint32_t own_b, uint32_t *indeg) {
+    for (unsigned long long e = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; e < E;
+         e += (unsigned long long)gridDim.x * blockDim.x)
+        atomicAdd(&indeg[col[e] - own_b], 1u);
 }
 
 __global__ void dist_sssp_init_kernel(unsigned long long *P, uint32_t *next_bm, uint32_t V, uint32_t gwords,
@@ -386,14 +430,25 @@ ag_status dist_sssp_scratch(ag_graph_s *g) {
     if (!g->d_P && (s = dev_alloc((void **)&g->d_P, (size_t)g->V * 8 + 128, g->device)) != AG_OK) return s;
     if (!d->d_send && (s = dev_alloc((void **)&d->d_send, (size_t)d->S * 8 + 128, g->device)) != AG_OK) return s;
     if (!d->d_list && (s = dev_alloc((void **)&d->d_list, (size_t)W * d->S * 8 + 128, g->device)) != AG_OK) return s;
-    if (!d->d_counts && (s = dev_alloc((void **)&d->d_counts, (size_t)W * 4 + 128, g->device)) != AG_OK) return s;
-    if (!d->h_counts && cudaMallocHost(&d->h_counts, (size_t)W * 4 + 64) != cudaSuccess)
+    if (!d->d_counts && (s = dev_alloc((void **)&d->d_counts, (size_t)W * CW * 4 + 128, g->device)) != AG_OK) return s;
+    if (!d->h_counts && cudaMallocHost(&d->h_counts, (size_t)W * CW * 4 + 64) != cudaSuccess)
         return set_error(AG_ERR_OOM, "pinned alloc");
+    for (int k = 0; k < 2; ++k)
+        if (!d->d_carry[k] && (s = dev_alloc((void **)&d->d_carry[k], (size_t)d->S * 4 + 128, g->device)) != AG_OK) return s;
+    if (!d->d_indeg) {
+        if ((s = dev_alloc((void **)&d->d_indeg, (size_t)d->S * 4 + 128, g->device)) != AG_OK) return s;
+        cudaMemset(d->d_indeg, 0, (size_t)d->S * 4 + 128);
+        if (g->E) dist_indeg_kernel<<<g->num_sms * 8, 256>>>(g->d_col, g->E, d->own_b, d->d_indeg);
+        note_launch(1);
+        cudaError_t e = cudaDeviceSynchronize();
+        if (e != cudaSuccess) return cuda_status(e, "in-degrees");
+    }
     return AG_OK;
 }
 
 template <typename Off>
-ag_status launch_sssp_round(ag_graph_s *g, const uint2 *list, uint32_t n, cudaStream_t st) {
+ag_status launch_sssp_round(ag_graph_s *g, const uint2 *list, uint32_t n, uint32_t ncin, int cpar,
+                            unsigned long long hi, cudaStream_t st) {
     ag_dist_part *d = g->dist;
     TravArgs<Off> a;
     memset(&a, 0, sizeof a);
@@ -421,15 +476,20 @@ ag_status launch_sssp_round(ag_graph_s *g, const uint2 *list, uint32_t n, cudaSt
     cudaError_t e = cudaLaunchCooperativeKernel((const void *)fn, dim3(a.nblocks), dim3(BS), args, 0, st);
     note_launch(1);
     if (e != cudaSuccess) return cuda_status(e, "dist sssp round");
-    dist_sssp_collect_kernel<<<g->num_sms * 2, 256, 0, st>>>(g->d_q[1], &((Ctl *)g->d_ctl)->q_len[1], g->d_P, d->d_next,
-                                                             d->d_send, d->d_counts + d->comm->rank);
+    unsigned *cnt = d->d_counts + (size_t)d->comm->rank * CW;
+    cudaMemsetAsync(cnt, 0, 8, st);
+    cudaMemsetAsync(cnt + 2, 0xFF, 4, st);
+    dist_sssp_collect_kernel<<<g->num_sms * 2, 256, 0, st>>>(d->d_carry[cpar], ncin, g->d_q[1], &((Ctl *)g->d_ctl)->q_len[1],
+                                                             g->d_P, d->d_indeg, d->own_b, hi, d->d_next, d->d_send,
+                                                             d->d_carry[cpar ^ 1], cnt);
     note_launch(1);
     return cuda_status(cudaGetLastError(), "dist sssp collect");
 }
 
-ag_status run_sssp_round(ag_graph_s *g, const uint2 *list, uint32_t n, cudaStream_t st) {
-    return g->offs32 ? launch_sssp_round<uint32_t>(g, list, n, st)
-                     : launch_sssp_round<unsigned long long>(g, list, n, st);
+ag_status run_sssp_round(ag_graph_s *g, const uint2 *list, uint32_t n, uint32_t ncin, int cpar, unsigned long long hi,
+                         cudaStream_t st) {
+    return g->offs32 ? launch_sssp_round<uint32_t>(g, list, n, ncin, cpar, hi, st)
+                     : launch_sssp_round<unsigned long long>(g, list, n, ncin, cpar, hi, st);
 }
 
 ag_status run_level(ag_graph_s *g, uint32_t L, uint32_t *parent_local, cudaStream_t st) {
@@ -720,7 +780,8 @@ ag_status dist_bfs_driver(std::vector<ag_graph_s *> &parts, uint32_t src, uint32
 // expands the same gathered list, collects its improved owned vertices, the per-rank counts are
 // all-gathered (termination: all zero), then the (v, dist) lists padded to the largest count.
 ag_status dist_sssp_driver(std::vector<ag_graph_s *> &parts, uint32_t src, uint32_t **dist_owned,
-                           uint32_t **parents_owned, ag_run_stats *stats, cudaStream_t st) {
+                           uint32_t **parents_owned, ag_run_stats *stats, cudaStream_t st,
+                           uint32_t hub_window) {
     const int P = (int)parts.size();
     ag_status s;
     for (auto *g : parts) {
@@ -751,37 +812,52 @@ ag_status dist_sssp_driver(std::vector<ag_graph_s *> &parts, uint32_t src, uint3
     uint32_t n = 1, R = 0;   // entries of the gathered list (with padding), rounds
     uint64_t front = 1;      // real entries
     const uint32_t tcap = stats ? stats->trace_cap : 0;
+    // owner-side hub window: hi = (global minimum pending distance) + hub_window; 0 = off (send all)
+    unsigned long long hi = hub_window ? (unsigned long long)hub_window : ~0ull;
+    int cpar = 0;                               // carry buffer read this round
+    std::vector<uint32_t> ncin(P, 0u);          // carried (held-back) entries per local part
     for (;; ++R) {
         if (stats && R < tcap && stats->trace_ws) stats->trace_ws[R] = (uint32_t)front;
-        for (auto *g : parts)
-            if ((s = run_sssp_round(g, g->dist->d_list, n, st)) != AG_OK) return s;
-        // counts: every rank's count to every rank
+        for (int r = 0; r < P; ++r)
+            if ((s = run_sssp_round(parts[r], parts[r]->dist->d_list, n, ncin[r], cpar, hi, st)) != AG_OK) return s;
+        // counts: every rank's (sent, carried, min pending) to every rank
         if (nccl) {
             ag_dist_part *d = parts[0]->dist;
-            ncclResult_t r = g_nccl.AllGather(d->d_counts + d->comm->rank, d->d_counts, 1, ncclUint32, d->comm->nccl, st);
+            ncclResult_t r = g_nccl.AllGather(d->d_counts + (size_t)d->comm->rank * CW, d->d_counts, CW, ncclUint32,
+                                              d->comm->nccl, st);
             if ((s = nccl_status(r, "ncclAllGather(counts)")) != AG_OK) return s;
         } else {
             for (auto *gd : parts)
                 for (auto *gs : parts)
                     if (gd != gs)
-                        cudaMemcpyAsync(gd->dist->d_counts + gs->dist->comm->rank, gs->dist->d_counts + gs->dist->comm->rank, 4,
+                        cudaMemcpyAsync(gd->dist->d_counts + (size_t)gs->dist->comm->rank * CW,
+                                        gs->dist->d_counts + (size_t)gs->dist->comm->rank * CW, CW * 4,
                                         cudaMemcpyDeviceToDevice, st);
         }
         ag_dist_part *d0 = parts[0]->dist;
-        cudaMemcpyAsync(d0->h_counts, d0->d_counts, (size_t)world * 4, cudaMemcpyDeviceToHost, st);
+        cudaMemcpyAsync(d0->h_counts, d0->d_counts, (size_t)world * CW * 4, cudaMemcpyDeviceToHost, st);
         cudaError_t ce = cudaStreamSynchronize(st);
         if (ce != cudaSuccess) return cuda_status(ce, "dist sssp round");
-        uint32_t maxc = 0;
+        uint32_t maxc = 0, lo = INF;
+        uint64_t carried = 0;
         front = 0;
         for (int r = 0; r < world; ++r) {
-            maxc = d0->h_counts[r] > maxc ? d0->h_counts[r] : maxc;
-            front += d0->h_counts[r];
+            const unsigned *c = d0->h_counts + (size_t)r * CW;
+            maxc = c[0] > maxc ? c[0] : maxc;
+            front += c[0];
+            carried += c[1];
+            lo = c[2] < lo ? c[2] : lo;
         }
-        if (front == 0 || R > 4u * V + 64u) break;
+        for (int r = 0; r < P; ++r) ncin[r] = d0->h_counts[(size_t)parts[r]->dist->comm->rank * CW + 1];
+        cpar ^= 1;
+        if (hub_window) hi = lo == INF ? ~0ull : (unsigned long long)lo + hub_window;
+        if ((front == 0 && carried == 0) || R > 4u * V + 64u) break;
+        n = (uint32_t)world * maxc;
+        if (maxc == 0) continue;   // everything pending is held back: next round sends the window's minimum
         // pad every send list to maxc with (INF, INF), then gather rank-ordered into the global list
         for (auto *g : parts) {
             ag_dist_part *d = g->dist;
-            const uint32_t c = d0->h_counts[d->comm->rank];
+            const uint32_t c = d0->h_counts[(size_t)d->comm->rank * CW];
             if (c < maxc) cudaMemsetAsync(d->d_send + c, 0xFF, (size_t)(maxc - c) * 8, st);
         }
         if (nccl) {
@@ -794,7 +870,6 @@ ag_status dist_sssp_driver(std::vector<ag_graph_s *> &parts, uint32_t src, uint3
                     cudaMemcpyAsync(gd->dist->d_list + (size_t)gs->dist->comm->rank * maxc, gs->dist->d_send,
                                     (size_t)maxc * 8, cudaMemcpyDeviceToDevice, st);
         }
-        n = (uint32_t)world * maxc;
     }
     for (int r = 0; r < P; ++r) {
         ag_graph_s *g = parts[r];
@@ -876,7 +951,6 @@ ag_status ag_dist_bfs_group(ag_graph *locals, int world, uint32_t src, uint32_t 
 
 ag_status ag_dist_sssp(ag_graph local, uint32_t src, uint32_t *dist_owned, uint32_t *parents_owned,
                        const ag_policy *policy, ag_run_stats *stats, void *stream) {
-    (void)policy;
     if (!local || !local->dist) return set_error(AG_ERR_INVALID_ARG, "not a distributed graph");
     if (!dist_owned) return set_error(AG_ERR_INVALID_ARG, "dist_owned is NULL");
     if (src >= local->V) return set_error(AG_ERR_SRC_RANGE, "src %u >= V %u", src, local->V);
@@ -886,7 +960,11 @@ ag_status ag_dist_sssp(ag_graph local, uint32_t src, uint32_t *dist_owned, uint3
     uint32_t *dv[1] = {dist_owned};
     uint32_t *pa[1] = {parents_owned};
     cudaSetDevice(local->device);
-    return dist_sssp_driver(parts, src, dv, parents_owned ? pa : nullptr, stats, (cudaStream_t)stream);
+    // owner-side hub window: policy->sssp_hub_window, AUTO = max(1, max weight / 50)
+    uint32_t hw = local->info.max_weight / 50u > 1u ? local->info.max_weight / 50u : 1u;
+    if (policy && policy->struct_size == sizeof(ag_policy) && policy->sssp_hub_window != AG_WINDOW_AUTO)
+        hw = policy->sssp_hub_window;
+    return dist_sssp_driver(parts, src, dv, parents_owned ? pa : nullptr, stats, (cudaStream_t)stream, hw);
 }
 
 ag_status ag_dist_sssp_group(ag_graph *locals, int world, uint32_t src, uint32_t **dist_owned,
@@ -901,7 +979,8 @@ ag_status ag_dist_sssp_group(ag_graph *locals, int world, uint32_t src, uint32_t
     if (src >= parts[0]->V) return set_error(AG_ERR_SRC_RANGE, "src out of range");
     if (stats && stats->struct_size != sizeof(ag_run_stats)) return set_error(AG_ERR_INVALID_ARG, "stats size");
     cudaSetDevice(parts[0]->device);
-    return dist_sssp_driver(parts, src, dist_owned, parents_owned, stats, (cudaStream_t)stream);
+    const uint32_t mw = parts[0]->info.max_weight;
+    return dist_sssp_driver(parts, src, dist_owned, parents_owned, stats, (cudaStream_t)stream, mw / 50u > 1u ? mw / 50u : 1u);
 }
 
 }  // extern "C"

@@ -187,8 +187,11 @@ def test_nccl_world1():
 # ------------------------------------------------------------------------------------------------
 def _partitioned_sssp_worker(rank, world, port, scale, src, out_q):
     """The distributed unordered SSSP of ag_dist_sssp on CPU: every rank relaxes the gathered global
-    list of (u, dist u) over its destination-owned part, then the improved owned vertices are
-    exchanged — all_gather of the counts, then of the (v, dist) lists padded to the largest count."""
+    list of (u, dist u) over its destination-owned part; the improved owned vertices join the rank's
+    pending set, from which the OWNER sends every non-hub (in-degree < 64) vertex and every hub below
+    hi = (global minimum pending distance of the last exchange) + hub window, holding the other hubs
+    back; all_gather of (sent, held back, min pending), then of the (v, dist) lists padded to the
+    largest count; done when nothing is sent or held back anywhere."""
     import torch
     import torch.distributed as dist
     from paper_conf_ipps_lib13_b200 import agraph as A
@@ -202,10 +205,13 @@ def _partitioned_sssp_worker(rank, world, port, scale, src, out_q):
     d = np.full(V, oracle.INF, np.int64)
     if b <= src < e:
         d[src] = 0
+    indeg = np.bincount(part.col.astype(np.int64) - b, minlength=max(e - b, 1))
+    hw = max(1, int(w.max()) // 50) if len(w) else 1
+    hi = hw
+    pending = set()
     lst = [(src, 0)]
     rounds = 0
     while True:
-        improved = set()
         for u, du in lst:
             for k in range(part.row_ptr[u], part.row_ptr[u + 1]):
                 v = int(part.col[k])
@@ -213,15 +219,23 @@ def _partitioned_sssp_worker(rank, world, port, scale, src, out_q):
                 nd = du + int(w[k])
                 if nd < d[v]:
                     d[v] = nd
-                    improved.add(v)
-        mine = sorted(improved)
-        cnt = torch.tensor([len(mine)], dtype=torch.int64)
-        counts = [torch.zeros(1, dtype=torch.int64) for _ in range(world)]
+                    pending.add(v)
+        lmin = min((int(d[v]) for v in pending), default=oracle.INF)
+        mine = sorted(v for v in pending if indeg[v - b] < 64 or d[v] < hi)
+        pending -= set(mine)
+        cnt = torch.tensor([len(mine), len(pending), lmin], dtype=torch.int64)
+        counts = [torch.zeros(3, dtype=torch.int64) for _ in range(world)]
         dist.all_gather(counts, cnt)
-        maxc = int(max(c.item() for c in counts))
+        maxc = int(max(c[0].item() for c in counts))
+        held = sum(int(c[1].item()) for c in counts)
+        lo = min(int(c[2].item()) for c in counts)
+        hi = lo + hw if lo != oracle.INF else 1 << 62
         rounds += 1
-        if maxc == 0:
+        if maxc == 0 and held == 0:
             break
+        if maxc == 0:
+            lst = []
+            continue
         buf = torch.full((maxc, 2), -1, dtype=torch.int64)
         for i, v in enumerate(mine):
             buf[i, 0], buf[i, 1] = v, int(d[v])
