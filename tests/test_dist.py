@@ -337,3 +337,33 @@ def test_nccl_world1_sssp():
         assert np.array_equal(d, ref)
     part.free()
     comm.free()
+
+
+@pytest.mark.gpu
+def test_c5_full_size_world8_virtual_group():
+    """C5 at full size (R-MAT scale 26, 2.1B CSR entries) partitioned 1-D over 8 ranks on one GPU: the
+    partition, kernels and exchange protocol of the 8-GPU bench (the all-gathers are device copies).
+    BFS levels are compared with
+    the oracle element by element; SSSP distances with parents must pass the shortest-path certificate
+    (edge inequalities + a tight parent edge for every reached vertex = exact distances)."""
+    import torch
+    from paper_conf_ipps_lib13_b200 import agraph as A
+    world = 8
+    g = aggen.config("C5")
+    # the global CSR goes to the device once; every rank keeps its destination-owned part of it
+    t = [torch.from_numpy(x.view(np.int64 if x.dtype == np.uint64 else np.int32)).cuda() for x in (g.row_ptr, g.col, g.w)]
+    comms = A.local_group(world, 0)
+    parts = [A.DistGraph(c, g.V, t[0], t[1], t[2]) for c in comms]
+    del t
+    torch.cuda.empty_cache()
+    src = int(aggen.sources(g, 1, seed=3)[0])
+    lv, _, _ = A.dist_bfs_group(parts, src)
+    ref, _ = oracle.bfs(g, src, want_parents=False)
+    assert np.array_equal(lv, ref)
+    d, par, _ = A.dist_sssp_group(parts, src, parents=True)
+    assert np.array_equal(d != oracle.INF, ref != oracle.INF)
+    assert oracle.validate(g, src, d, par, weighted=True)[0] == 0
+    for p in parts:
+        p.free()
+    for c in comms:
+        c.free()
