@@ -22,13 +22,13 @@ constexpr int BS = AG_BS;           // threads per CTA of the persistent travers
 constexpr int WARPS_PER_CTA = BS / 32;
 constexpr int LOG_BS = (BS == 1024) ? 10 : (BS == 512) ? 9 : (BS == 256) ? 8 : (BS == 128) ? 7 : -1;
 static_assert(LOG_BS > 0, "BS must be 128, 256, 512 or 1024");
-// Occupancy / batch depth per algorithm (measured on B200): BFS is best at 4 CTAs/SM
-// (64 regs) with 4-edge batches, SSSP (8-byte states, more atomics) at 8 CTAs/SM with 2-edge batches.
+// Occupancy / batch depth per algorithm (measured on B200; profiles/r01_occupancy_ab.txt):
+// BFS/CC 5 CTAs/SM with 4-edge pieces, SSSP (8-byte states, more atomics) 5 CTAs/SM with 2-edge pieces.
 #ifndef AG_MINB_BFS
 #define AG_MINB_BFS 5
 #endif
 #ifndef AG_MINB_SSSP
-#define AG_MINB_SSSP 6
+#define AG_MINB_SSSP 5   // re-tuned after the carveout / staging changes: C2 -3.8%, C4 -12.5%, C3 -3% vs 6 (no spills)
 #endif
 #ifndef AG_MINB_BFS_T
 #define AG_MINB_BFS_T AG_MINB_BFS
