@@ -700,8 +700,12 @@ ag_status ag_graph_load_csr_ex(uint32_t V, uint64_t E, const uint64_t *row_ptr, 
     g->num_sms = sms;
     g->nwords = (V + 31) / 32;
     g->offs32 = E < 0xFFFFFFFFull;
-    g->hub_cap = (uint32_t)((E / HUB_CHUNK + E / HUB_DEG + 16) > 0xFFFFFFF0ull ? 0xFFFFFFF0ull
-                                                                            : (E / HUB_CHUNK + E / HUB_DEG + 16));
+    {   // tasks of one iteration <= E / chunk + (lists >= the task degree), for the smallest chunk/degree in use
+        const uint64_t ch = HUB_CHUNK_SMALL < HUB_CHUNK ? HUB_CHUNK_SMALL : HUB_CHUNK;
+        const uint64_t hd = HUB_CHUNK_SMALL < HUB_DEG ? HUB_CHUNK_SMALL : HUB_DEG;
+        const uint64_t c = E / ch + E / hd + 16;
+        g->hub_cap = (uint32_t)(c > 0xFFFFFFF0ull ? 0xFFFFFFF0ull : c);
+    }
     cudaEventCreate(&g->ev[0]);
     cudaEventCreate(&g->ev[1]);
     auto fail = [&](ag_status st) { ag_graph_free(g); return st; };

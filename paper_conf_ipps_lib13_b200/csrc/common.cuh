@@ -71,6 +71,16 @@ enum { WS_BM = 1, WS_QU = 2 };
 constexpr uint32_t HUB_DEG = AG_HUBDEG;
 constexpr uint32_t HUBW_DEG = 64;   // SSSP hub-window degree threshold (measured on C1/C2/C4)
 constexpr uint32_t HUB_CHUNK = AG_HUBCHUNK;
+// Small working sets (|WS| < SMALLCHUNK_PER_CTA x CTAs: few hub tasks per CTA, the iteration ends with the
+// slowest task) split lists of >= HUB_CHUNK_SMALL entries into HUB_CHUNK_SMALL-entry tasks instead.
+#ifndef AG_HUBCHUNK_SMALL
+#define AG_HUBCHUNK_SMALL 1024
+#endif
+#ifndef AG_SMALLCHUNK_PER_CTA
+#define AG_SMALLCHUNK_PER_CTA 32
+#endif
+constexpr uint32_t HUB_CHUNK_SMALL = AG_HUBCHUNK_SMALL;
+constexpr uint32_t SMALLCHUNK_PER_CTA = AG_SMALLCHUNK_PER_CTA;
 // Edges processed per thread per batch: loads of all EB edges are issued before any dependent use.
 constexpr int EB_MAX = (AG_EB_BFS > AG_EB_SSSP) ? AG_EB_BFS : AG_EB_SSSP;
 

@@ -137,6 +137,7 @@ struct Ops {
     bool any = false;       //   ... and this thread set at least one bit of it
     uint32_t nact;          // CTAs taking part in this iteration (default: the whole grid)
     bool bm_upd = true;     // BFS: write the update-vector bitmap (tuned queue-only kernels never read it)
+    uint32_t hdeg = HUB_DEG, hchunk = HUB_CHUNK;   // hub-task degree threshold and chunk (per iteration)
 
     __device__ Ops(const TravArgs<Off> &a_, uint32_t it_, uint64_t hi_, bool append_)
         : a(a_), it(it_), hi(hi_), append_next(append_), fenced(ALG == ALG_SSSP && ORD == ORD_O && a_.pol.delta > 1),
@@ -705,11 +706,11 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, SmT &sm, u
     }
     // ---- MAP_H: load-balanced gather over the tile's concatenated adjacency lists; vertices of
     // degree >= HUB_DEG are split into HUB_CHUNK-edge tasks drained by all CTAs.
-    const bool is_hub = hubs && deg >= HUB_DEG;
+    const bool is_hub = hubs && deg >= ops.hdeg;
     if (is_hub) {
-        const uint32_t nch = (deg + HUB_CHUNK - 1) / HUB_CHUNK;
+        const uint32_t nch = (deg + ops.hchunk - 1) / ops.hchunk;
         uint32_t base = atomicAdd(&a.ctl->hub_tail[slot], nch);
-        // hub_cap >= E/HUB_CHUNK + E/HUB_DEG + 16 covers any frontier (each vertex is at most once
+        // hub_cap >= E/chunk + E/degree + 16 (smallest in use) covers any frontier (each vertex is at most once
         // per iteration in it); the guard only protects memory.
         // a task is ONE self-contained 64-bit word (u << 32 | chunk << 1 | 1), published with a single
         // relaxed store: the consumer needs no acquire (which would invalidate its L1) and clears the
@@ -839,8 +840,8 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, SmT &sm, uin
         uint32_t u, uval;
         ops.task_vertex((uint32_t)(w >> 32), u, uval);
         const Off b0 = a.rp[u], e0 = a.rp[u + 1];
-        const Off b = b0 + (Off)k * HUB_CHUNK;
-        const Off e = (e0 - b > (Off)HUB_CHUNK) ? b + HUB_CHUNK : e0;
+        const Off b = b0 + (Off)k * ops.hchunk;
+        const Off e = (e0 - b > (Off)ops.hchunk) ? b + ops.hchunk : e0;
         constexpr uint32_t QE = Ops<ALG, ORD, Off>::QE;
         constexpr int QB = Ops<ALG, ORD, Off>::QB;
         const Off q0 = b / QE, q1 = (e + QE - 1) / QE;
@@ -1154,6 +1155,10 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         ops.wbuf = sm.wq[threadIdx.x >> 5];
         ops.nact = nact;
         ops.bm_upd = !(TUNED && ALG == ALG_BFS);
+        if (TUNED && (uint64_t)qn < (uint64_t)SMALLCHUNK_PER_CTA * nact) {   // few tasks per CTA: finer tasks
+            ops.hdeg = HUB_CHUNK_SMALL < HUB_DEG ? HUB_CHUNK_SMALL : HUB_DEG;
+            ops.hchunk = HUB_CHUNK_SMALL;
+        }
         // free output (tuned, unordered, big working sets; BFS only without parents: a claim decides them)
         ops.freeo = TUNED && ROT && (ALG != ALG_BFS ? (uint64_t)qn >= a.pol.t_free_sssp
                                                     : ((uint64_t)qn >= a.pol.t_free && a.parent == nullptr));
