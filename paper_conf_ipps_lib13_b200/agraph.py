@@ -401,8 +401,7 @@ def use_torch_allocator(enable: bool = True):
     L.ag_set_allocator.argtypes = [_ALLOC_T, _FREE_T, ctypes.c_void_p]
     if not enable:
         _check(L.ag_set_allocator(_ALLOC_T(0), _FREE_T(0), None))
-        _alloc_refs = None
-        return
+        return   # (the callbacks stay referenced: buffers allocated through them are freed through them)
     import torch
 
     def _alloc(nbytes, dev, stream, ctx):
@@ -414,5 +413,6 @@ def use_torch_allocator(enable: bool = True):
     def _free(ptr, nbytes, dev, stream, ctx):
         torch.cuda.caching_allocator_delete(int(ptr))
 
-    _alloc_refs = (_ALLOC_T(_alloc), _FREE_T(_free))
-    _check(L.ag_set_allocator(_alloc_refs[0], _alloc_refs[1], None))
+    refs = (_ALLOC_T(_alloc), _FREE_T(_free))
+    _alloc_refs = (_alloc_refs or []) + [refs]
+    _check(L.ag_set_allocator(refs[0], refs[1], None))

@@ -9,6 +9,7 @@
 #include <cstring>
 #include <mutex>
 #include <string>
+#include <unordered_map>
 #include <vector>
 
 #include <cub/device/device_radix_sort.cuh>
@@ -53,13 +54,26 @@ static void *(*g_alloc)(size_t, int, void *, void *) = nullptr;
 static void (*g_free)(void *, size_t, int, void *, void *) = nullptr;
 static void *g_alloc_ctx = nullptr;
 
+// Every hook allocation remembers the free function that owns it, so a buffer is always returned to the
+// allocator it came from — also when the hook is changed or removed between allocation and free (a
+// graph loaded with cudaMalloc and freed while the PyTorch hook is active, or the reverse).
+struct HookRec {
+    void (*free_)(void *, size_t, int, void *, void *);
+    void *ctx;
+};
+static std::unordered_map<void *, HookRec> g_hook_ptrs;
+static std::mutex g_hook_mu;
+
 ag_status dev_alloc(void **p, size_t bytes, int device) {
     *p = nullptr;
     if (bytes == 0) bytes = 16;
     bytes = (bytes + 255) & ~size_t(255);
     if (g_alloc) {
         *p = g_alloc(bytes, device, nullptr, g_alloc_ctx);
-        return *p ? AG_OK : set_error(AG_ERR_OOM, "allocator hook returned NULL for %zu bytes", bytes);
+        if (!*p) return set_error(AG_ERR_OOM, "allocator hook returned NULL for %zu bytes", bytes);
+        std::lock_guard<std::mutex> lk(g_hook_mu);
+        g_hook_ptrs[*p] = HookRec{g_free, g_alloc_ctx};
+        return AG_OK;
     }
     return cuda_status(cudaMalloc(p, bytes), "cudaMalloc");
 }
@@ -67,7 +81,16 @@ ag_status dev_alloc(void **p, size_t bytes, int device) {
 void dev_free(void *p, size_t bytes, int device) {
     if (!p) return;
     bytes = (bytes == 0 ? 16 : (bytes + 255) & ~size_t(255));
-    if (g_free) g_free(p, bytes, device, nullptr, g_alloc_ctx);
+    HookRec r{nullptr, nullptr};
+    {
+        std::lock_guard<std::mutex> lk(g_hook_mu);
+        auto it = g_hook_ptrs.find(p);
+        if (it != g_hook_ptrs.end()) {
+            r = it->second;
+            g_hook_ptrs.erase(it);
+        }
+    }
+    if (r.free_) r.free_(p, bytes, device, nullptr, r.ctx);
     else cudaFree(p);
 }
 

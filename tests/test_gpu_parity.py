@@ -422,3 +422,30 @@ def test_pipelined_load_degree_layout_edge_cases():
         if weighted:
             assert np.array_equal(G.sssp(0)[0], oracle.dijkstra(g, 0)[0])
         assert np.array_equal(G.cc()[0], oracle.cc(g))
+
+
+def test_allocator_hook_switched_between_load_and_free():
+    """A buffer always goes back to the allocator it came from, whatever the hook is at free time."""
+    import sys
+
+    import torch
+    errs = []
+    old = sys.unraisablehook
+    sys.unraisablehook = errs.append
+    try:
+        g = aggen.config("C1")
+        s = int(aggen.sources(g, 1)[0])
+        G1 = A.Graph.from_csr(g)                 # cudaMalloc
+        G1.bfs(s)
+        A.use_torch_allocator(True)
+        G2 = A.Graph.from_csr(g)                 # PyTorch caching allocator
+        G2.sssp(s)
+        G1.free()                                # -> cudaFree, not the torch hook
+        before = torch.cuda.memory_allocated()
+        A.use_torch_allocator(False)
+        G2.free()                                # -> back to torch although the hook is off
+        assert torch.cuda.memory_allocated() < before
+    finally:
+        A.use_torch_allocator(False)
+        sys.unraisablehook = old
+    assert not errs, errs
