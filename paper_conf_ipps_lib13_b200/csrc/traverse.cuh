@@ -81,6 +81,9 @@ struct TravArgs {
                                 // travels with the entry, hub tasks carry the entry index (nullptr: off)
 };
 
+#ifndef AG_BLIND
+#define AG_BLIND 1
+#endif
 // per-warp staging capacity: one batch appends at most 32 x (edges per thread per batch), plus < 32 left over
 // (sized per algorithm: the smaller SSSP buffer lets the L1/shared carveout leave more L1 to the status
 // gathers, see launch_traverse)
@@ -447,7 +450,13 @@ struct Ops {
                                                const uint32_t (&wt)[NB], const bool (&ok)[NB]) {
         St st[NB];
 #pragma unroll
-        for (int j = 0; j < NB; ++j) st[j] = ok[j] ? status(v[j]) : (St)0;
+        for (int j = 0; j < NB; ++j) {
+            // free-output BFS: no status gather — every target is marked with one fire-and-forget red.or
+            // and the next iteration's compaction drops the visited ones (one L2 operation per edge with
+            // no round trip, instead of a gather plus a red.or per unvisited target)
+            if (AG_BLIND && ALG == ALG_BFS && freeo) st[j] = (St)0;
+            else st[j] = ok[j] ? status(v[j]) : (St)0;
+        }
         if constexpr (STAGED) {
             const uint32_t nwm = update_batch<NB, true>(u, uv, v, wt, st, ok);  // bit j: v[j] entered the next WS
             if (__any_sync(0xffffffffu, nwm != 0)) {   // rare on the big levels: skip the ballots otherwise
