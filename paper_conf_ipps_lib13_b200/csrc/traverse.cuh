@@ -923,13 +923,27 @@ __device__ __forceinline__ void compact_raw(const TravArgs<Off> &a, SmT &sm, uin
             sm.bcast = tot ? atomicAdd(qlen, tot) : 0u;
         }
         __syncthreads();
-        uint32_t pos = sm.bcast + sm.red32[1][wid] + x - c;
-        while (word) {
-            const int b = __ffs(word) - 1;
-            word &= word - 1;
-            const uint32_t v = wi * 32 + b;
-            q[pos++] = v;
-            if constexpr (ALG == ALG_BFS) a.level[v] = lvl;   // m.level = level (Fig. 4 l.9)
+        // warp-cooperative emission, in order: output i of this warp goes to lane i % 32, which finds the
+        // owning word (binary search over the lanes' inclusive counts, by shuffles) and its bit (n-th set
+        // bit), so the queue and level stores of a warp are consecutive instead of one lane writing its
+        // whole word's run (32 scattered sectors per store instruction)
+        const uint32_t wbase = sm.bcast + sm.red32[1][wid], wtot = __shfl_sync(0xffffffffu, x, 31);
+        for (uint32_t i0 = 0; i0 < wtot; i0 += 32) {
+            const uint32_t i = i0 + lane;
+            uint32_t o = 0;   // first lane whose inclusive count exceeds i
+#pragma unroll
+            for (uint32_t step = 16; step >= 1; step >>= 1) {
+                const uint32_t xs = __shfl_sync(0xffffffffu, x, o + step - 1);
+                if (xs <= i) o += step;
+            }
+            o = o > 31u ? 31u : o;
+            const uint32_t ow = __shfl_sync(0xffffffffu, word, o);
+            const uint32_t oe = __shfl_sync(0xffffffffu, x - c, o);
+            if (i < wtot) {
+                const uint32_t v = (w0 + (wid << 5) + o) * 32u + __fns(ow, 0u, (int)(i - oe) + 1);
+                q[wbase + i] = v;
+                if constexpr (ALG == ALG_BFS) a.level[v] = lvl;   // m.level = level (Fig. 4 l.9)
+            }
         }
         __syncthreads();   // red32 / bcast reuse
     }
