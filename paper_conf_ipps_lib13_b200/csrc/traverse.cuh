@@ -884,6 +884,37 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, SmT &sm, uin
     }
 }
 
+// Warp-cooperative, in-order emission of the set bits of the warp's 32 consecutive words (word w0 + lane,
+// popcount c, inclusive warp count x, warp total tot) as vertex ids out[0 .. tot): output i goes to lane
+// i % 32, which finds the owning word (binary search over the lanes' inclusive counts, by shuffles) and
+// its bit (n-th set bit), so the warp's stores are consecutive instead of one lane writing its word's run
+// (32 scattered sectors per store instruction).  f(v) is called for every emitted vertex.
+template <typename F>
+__device__ __forceinline__ void warp_emit_f(uint32_t *out, uint32_t x, uint32_t c, uint32_t word, uint32_t w0,
+                                            uint32_t tot, F f) {
+    const uint32_t lane = lane_id();
+    for (uint32_t i0 = 0; i0 < tot; i0 += 32) {
+        const uint32_t i = i0 + lane;
+        uint32_t o = 0;   // first lane whose inclusive count exceeds i
+#pragma unroll
+        for (uint32_t step = 16; step >= 1; step >>= 1) {
+            const uint32_t xs = __shfl_sync(0xffffffffu, x, o + step - 1);
+            if (xs <= i) o += step;
+        }
+        o = o > 31u ? 31u : o;
+        const uint32_t ow = __shfl_sync(0xffffffffu, word, o);
+        const uint32_t oe = __shfl_sync(0xffffffffu, x - c, o);
+        if (i < tot) {
+            const uint32_t v = (w0 + o) * 32u + __fns(ow, 0u, (int)(i - oe) + 1);
+            out[i] = v;
+            f(v);
+        }
+    }
+}
+__device__ __forceinline__ void warp_emit(uint32_t *out, uint32_t x, uint32_t c, uint32_t word, uint32_t w0, uint32_t tot) {
+    warp_emit_f(out, x, c, word, w0, tot, [](uint32_t) {});
+}
+
 // Free-output successor -> queue: O(V/32) compaction of the raw next bitmap (the "converted in
 // O(V/32)" working-set switch; prefix scan instead of per-element atomics, 22.s24).  Each thread
 // takes one word per step, one atomic per CTA step.  BFS keeps only the unvisited bits, marks them
@@ -923,28 +954,10 @@ __device__ __forceinline__ void compact_raw(const TravArgs<Off> &a, SmT &sm, uin
             sm.bcast = tot ? atomicAdd(qlen, tot) : 0u;
         }
         __syncthreads();
-        // warp-cooperative emission, in order: output i of this warp goes to lane i % 32, which finds the
-        // owning word (binary search over the lanes' inclusive counts, by shuffles) and its bit (n-th set
-        // bit), so the queue and level stores of a warp are consecutive instead of one lane writing its
-        // whole word's run (32 scattered sectors per store instruction)
         const uint32_t wbase = sm.bcast + sm.red32[1][wid], wtot = __shfl_sync(0xffffffffu, x, 31);
-        for (uint32_t i0 = 0; i0 < wtot; i0 += 32) {
-            const uint32_t i = i0 + lane;
-            uint32_t o = 0;   // first lane whose inclusive count exceeds i
-#pragma unroll
-            for (uint32_t step = 16; step >= 1; step >>= 1) {
-                const uint32_t xs = __shfl_sync(0xffffffffu, x, o + step - 1);
-                if (xs <= i) o += step;
-            }
-            o = o > 31u ? 31u : o;
-            const uint32_t ow = __shfl_sync(0xffffffffu, word, o);
-            const uint32_t oe = __shfl_sync(0xffffffffu, x - c, o);
-            if (i < wtot) {
-                const uint32_t v = (w0 + (wid << 5) + o) * 32u + __fns(ow, 0u, (int)(i - oe) + 1);
-                q[wbase + i] = v;
-                if constexpr (ALG == ALG_BFS) a.level[v] = lvl;   // m.level = level (Fig. 4 l.9)
-            }
-        }
+        warp_emit_f(q + wbase, x, c, word, w0 + (wid << 5), wtot, [&](uint32_t v) {
+            if constexpr (ALG == ALG_BFS) a.level[v] = lvl;   // m.level = level (Fig. 4 l.9)
+        });
         __syncthreads();   // red32 / bcast reuse
     }
 }
@@ -968,12 +981,7 @@ __device__ __forceinline__ void compact_bitmap(const uint32_t *bm, uint32_t nwor
         uint32_t base = 0;
         if (lane == 31) base = atomicAdd(qlen, total);
         base = __shfl_sync(0xffffffffu, base, 31);
-        uint32_t pos = base + x - c;
-        while (word) {
-            int b = __ffs(word) - 1;
-            word &= word - 1;
-            q[pos++] = wi * 32 + b;
-        }
+        warp_emit(q + base, x, c, word, w0, total);
     }
 }
 
