@@ -22,12 +22,14 @@ import aggen  # noqa: E402
 from paper_conf_ipps_lib13_b200 import agraph as A  # noqa: E402
 
 
-def variants(orders):
+def variants(orders, kinds=(1,)):
     out = []
     for o in orders:
-        for m in (1, 2, 3, 4):
-            for w in (1, 2):
-                out.append((f"{'O' if o else 'U'}_{A.MAP_LETTER[m]}_{A.WS_NAME[w]}", dict(order=o, mapping=m, workset=w)))
+        for k in kinds:
+            for m in (1, 2, 3, 4):
+                for w in (1, 2):
+                    name = f"{'O' if o else 'U'}_{A.MAP_LETTER[m]}_{A.WS_NAME[w]}" + ("" if k == 1 else "_paper")
+                    out.append((name, dict(order=o, mapping=m, workset=w, kind=k)))
         out.append((f"{'O' if o else 'U'}_adaptive_paper", dict(order=o, kind=0)))
         out.append((f"{'O' if o else 'U'}_adaptive_tuned", dict(order=o, kind=1)))
     return out
@@ -39,6 +41,7 @@ def main():
     ap.add_argument("--sources", type=int, default=4)
     ap.add_argument("--alg", default="bfs,sssp")
     ap.add_argument("--orders", default="0,1")
+    ap.add_argument("--kinds", default="1", help="policy kinds of the static variants: 0 paper kernels, 1 tuned")
     ap.add_argument("--trace", action="store_true")
     ap.add_argument("--only", default="")
     ap.add_argument("--reps", type=int, default=2)
@@ -51,7 +54,8 @@ def main():
     extra = dict(kv.split("=") for kv in args.set.split(",") if kv)
     print(json.dumps({"config": args.config, "V": g.V, "E": g.E, "max_deg": G.info.max_deg}), flush=True)
     for alg in args.alg.split(","):
-        for name, kw in variants([int(x) for x in args.orders.split(",")]):
+        for name, kw in variants([int(x) for x in args.orders.split(",")],
+                                 [int(x) for x in args.kinds.split(",")]):
             if args.only and not any(t in name for t in args.only.split(",")):
                 continue
             if alg == "bfs" and kw.get("order") == 1 and False:
