@@ -6,7 +6,7 @@
 set -u
 mkdir -p gpurun_out/sweeps
 for cfg in ${CONFIGS:-C2 C4 C3}; do
-  timeout "${PER_CONFIG_S:-600}" python tools/sweep.py --config "$cfg" --sources 2 --reps 1 --orders 0,1 --kinds 0,1 \
+  timeout "${PER_CONFIG_S:-600}" python tools/sweep.py --config "$cfg" --sources ${SOURCES:-2} --reps ${REPS:-2} --orders 0,1 --kinds 0,1 \
     > "gpurun_out/sweeps/r01_static_${cfg}.jsonl" 2> "gpurun_out/sweeps/r01_static_${cfg}.err"
   echo "$cfg rc=$?"
 done
