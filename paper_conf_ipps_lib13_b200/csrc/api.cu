@@ -383,6 +383,8 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
     if (const char *ts = getenv("AG_SMALL_WS")) d.t_small = (uint32_t)atoi(ts);   // experiments / tests
     d.t_small_hub = p.kind == AG_POLICY_TUNED ? 4096u : 0u;   // C2: BFS -1.6%, SSSP -2.7% (median of 12)
     if (const char *ts = getenv("AG_SMALL_HUB_WS")) d.t_small_hub = (uint32_t)atoi(ts);
+    d.smallchunk_per_cta = SMALLCHUNK_PER_CTA;
+    if (const char *ts = getenv("AG_SMALLCHUNK_PER_CTA")) d.smallchunk_per_cta = (uint32_t)atoi(ts);   // experiments
     return d;
 }
 

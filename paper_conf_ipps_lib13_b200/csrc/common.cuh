@@ -144,6 +144,7 @@ struct DevPolicy {
     uint32_t small_ctas;  // tuned kernels: CTAs that run an iteration whose |WS| < t_small (the rest park)
     uint32_t t_small;     //   0 = off
     uint32_t t_small_hub; //   graphs with hub tasks: only in the shrinking tail (|WS| below this and falling)
+    uint32_t smallchunk_per_cta;  // tuned kernels: |WS| < this x CTAs -> HUB_CHUNK_SMALL-entry hub tasks
 };
 
 // The decision maker.  PAPER: Fig. 11 with readings R12/R13:

@@ -1186,7 +1186,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         ops.wbuf = sm.wq[threadIdx.x >> 5];
         ops.nact = nact;
         ops.bm_upd = !(TUNED && ALG == ALG_BFS);
-        if (TUNED && (uint64_t)qn < (uint64_t)SMALLCHUNK_PER_CTA * nact) {   // few tasks per CTA: finer tasks
+        if (TUNED && (uint64_t)qn < (uint64_t)a.pol.smallchunk_per_cta * nact) {   // few tasks per CTA: finer tasks
             ops.hdeg = HUB_CHUNK_SMALL < HUB_DEG ? HUB_CHUNK_SMALL : HUB_DEG;
             ops.hchunk = HUB_CHUNK_SMALL;
         }
