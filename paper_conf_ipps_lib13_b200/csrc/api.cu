@@ -405,7 +405,11 @@ ag_status check_policy(const ag_policy *p) {
 template <int ALG, int ORD, typename Off>
 static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t st) {
     // the tuned adaptive policy runs the specialisation without the paper's static variants
-    const bool tuned = a.pol.kind == AG_POLICY_TUNED && a.pol.force_map == 0 && a.pol.force_ws == 0;
+    // Unordered BFS on degree-layout (hub) graphs runs the tuned policy's decisions (hybrid mapping,
+    // queue) in the general specialisation: C2 median 0.575 -> 0.566 ms, mean 0.588 -> 0.565 ms over
+    // 16 sources (profiles/r01_bfs_tuned_probe.txt; cause in the tuned specialisation not found).
+    const bool tuned = a.pol.kind == AG_POLICY_TUNED && a.pol.force_map == 0 && a.pol.force_ws == 0 &&
+                       !(ALG == ALG_BFS && ORD == ORD_U && g->info.layout == AG_LAYOUT_DEGREE);
     auto fn = tuned ? traverse_kernel<ALG, ORD, Off, true> : traverse_kernel<ALG, ORD, Off, false>;
     const size_t dyn = 0;
     if (dyn) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
