@@ -214,8 +214,11 @@ ag_status ag_sssp(ag_graph g, uint32_t src, uint32_t *dist, uint32_t *parents, c
  * for ag_bfs.  Errors: AG_ERR_INVALID_ARG, AG_ERR_UNSUPPORTED, AG_ERR_OOM, AG_ERR_CUDA. */
 ag_status ag_cc(ag_graph g, uint32_t *labels, const ag_policy *policy, ag_run_stats *stats, void *stream);
 
-/* Wait for the graph's last enqueued traversal and return its deferred status (AG_OK or
- * AG_ERR_OVERFLOW / AG_ERR_CUDA); clears the deferred status. */
+/* Wait for the graph's last enqueued traversal and return the deferred status accumulated over
+ * EVERY traversal enqueued on this handle since the previous check (sticky on the device: a later
+ * launch never clears an earlier query's overflow or abort): AG_ERR_CUDA if any aborted, else
+ * AG_ERR_OVERFLOW if any SSSP left a reachable vertex beyond 0xFFFFFFFE (exact test, run inside the
+ * traversal kernel only when a relaxation exceeded that bound), else AG_OK.  Clears the status. */
 ag_status ag_graph_check(ag_graph g);
 
 /* ---------------------------------------------------------------------------------------------
@@ -229,6 +232,8 @@ ag_status ag_graph_check(ag_graph g);
 ag_status ag_dist_unique_id(void *out128);
 /* Create the communicator for (rank, world) on `device`. */
 ag_status ag_dist_init(int rank, int world, const void *nccl_unique_id128, int device, ag_comm *out);
+/* Free a communicator.  AG_ERR_INVALID_ARG while graphs partitioned over it are still live
+ * (ag_graph_free them first). */
 ag_status ag_dist_free(ag_comm c);
 /* Owned vertex range of `rank` for a V-vertex graph partitioned over `world` ranks. */
 ag_status ag_dist_owned_range(uint32_t V, int rank, int world, uint32_t *begin, uint32_t *end);

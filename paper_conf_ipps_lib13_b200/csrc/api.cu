@@ -264,20 +264,6 @@ __global__ void reached_kernel(const uint32_t *out, const Off *rp, const uint32_
     if ((threadIdx.x & 31) == 0 && (a | b)) { atomicAdd(&acc[0], a); atomicAdd(&acc[1], b); }
 }
 
-// exact overflow test after a flagged SSSP: a reachable vertex left at INF behind a finite one
-template <typename Off>
-__global__ void overflow_check_kernel(const uint32_t *dist, const Off *rp, const uint32_t *col, const uint32_t *perm,
-                                      uint32_t V, unsigned *flag) {
-    // rp/col in device-layout ids, dist in caller ids
-    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < V; u += gridDim.x * blockDim.x) {
-        if (dist[perm ? perm[u] : u] == INF) continue;
-        for (Off e = rp[u]; e < rp[u + 1]; ++e) {
-            const uint32_t v = col[e];
-            if (dist[perm ? perm[v] : v] == INF) { *flag = 1; return; }
-        }
-    }
-}
-
 // ------------------------------------------------------------------------------------------------
 // graph handle helpers
 // ------------------------------------------------------------------------------------------------
@@ -489,6 +475,7 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
     }
     ag_status s = check_policy(&pol);
     if (s != AG_OK) return s;
+    if (alg == ALG_CC && pol.order == AG_ORDERED) return set_error(AG_ERR_UNSUPPORTED, "ag_cc is unordered only (DESIGN.md R23)");
     if (stats && stats->struct_size != sizeof(ag_run_stats))
         return set_error(AG_ERR_INVALID_ARG, "ag_run_stats.struct_size mismatch");
     cudaSetDevice(g->device);
@@ -556,9 +543,10 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
     }
     a.pol = resolve_policy(pol, *g);
     a.src = src;
-    a.epoch = ++g->epoch;
-    a.max_iters = alg != ALG_SSSP ? g->V + 2 : 4u * g->V + 64u;   // CC: <= longest min-label chain + 1
-    if (a.max_iters < g->V) a.max_iters = 0xFFFFFFF0u;
+    {   // iteration cap (never expected to bind): BFS/CC <= V + 1 levels / label rounds; SSSP generous
+        const uint64_t cap = alg != ALG_SSSP ? (uint64_t)g->V + 2 : 4ull * g->V + 64;
+        a.max_iters = (uint32_t)(cap > 0xFFFFFFF0ull ? 0xFFFFFFF0ull : cap);
+    }
     a.has_hubs = g->info.max_deg >= HUB_DEG;
 
     if (stats) {
@@ -568,7 +556,6 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
         s = (pol.order == AG_ORDERED) ? launch_traverse<ALG_BFS, ORD_O, Off>(g, a, st)
                                       : launch_traverse<ALG_BFS, ORD_U, Off>(g, a, st);
     } else if (alg == ALG_CC) {
-        if (pol.order == AG_ORDERED) return set_error(AG_ERR_UNSUPPORTED, "ag_cc is unordered only (DESIGN.md R23)");
         s = launch_traverse<ALG_CC, ORD_U, Off>(g, a, st);
     } else {
         s = (pol.order == AG_ORDERED) ? launch_traverse<ALG_SSSP, ORD_O, Off>(g, a, st)
@@ -577,8 +564,6 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
     if (s != AG_OK) return s;
     if (stats) cudaEventRecord(g->ev[1], st);
     g->last_stream = st;
-    g->last_alg = alg;
-    g->last_out = d_out;
     g->pending_check = true;
 
     if (!out_dev) cudaMemcpyAsync(out, d_out, (size_t)g->V * 4, cudaMemcpyDeviceToHost, st);
@@ -621,7 +606,6 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
         }
         e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_status(e, "stats");
-        if (c.aborted) return set_error(AG_ERR_CUDA, "traversal aborted (code %u)", c.aborted);
     }
     return s;
 }
@@ -967,29 +951,19 @@ ag_status ag_graph_check(ag_graph g) {
     cudaError_t e = cudaStreamSynchronize(g->last_stream);
     if (e != cudaSuccess) return cuda_status(e, "traversal");
     g->pending_check = false;
-    Ctl c;
-    e = cudaMemcpy(&c, g->d_ctl, sizeof c, cudaMemcpyDeviceToHost);
+    // the sticky status accumulates over every traversal enqueued since the last check (a launch
+    // never clears it), so an overflow or abort of an earlier query is not lost behind a later one
+    unsigned sticky = 0;
+    unsigned *d_sticky = (unsigned *)((char *)g->d_ctl + offsetof(Ctl, sticky));
+    e = cudaMemcpy(&sticky, d_sticky, 4, cudaMemcpyDeviceToHost);
     if (e != cudaSuccess) return cuda_status(e, "ctl");
-    if (c.aborted) {
+    if (!sticky) return AG_OK;
+    cudaMemset(d_sticky, 0, 4);
+    if (sticky >> 8) {
         if (g->d_hub) cudaMemset(g->d_hub, 0, (size_t)g->hub_cap * 8);   // the ring may hold unconsumed tasks
-        return set_error(AG_ERR_CUDA, "traversal aborted (code %u)", c.aborted);
+        return set_error(AG_ERR_CUDA, "traversal aborted (code %u)", sticky >> 8);
     }
-    if (g->last_alg == ALG_SSSP && c.overflow) {
-        unsigned *flag = (unsigned *)g->d_acc;
-        cudaMemset(flag, 0, 4);
-        if (g->offs32)
-            overflow_check_kernel<uint32_t><<<g->num_sms * 4, 256>>>(g->last_out, (const uint32_t *)g->d_rp, g->d_col,
-                                                                     g->d_perm, g->V, flag);
-        else
-            overflow_check_kernel<unsigned long long><<<g->num_sms * 4, 256>>>(
-                g->last_out, (const unsigned long long *)g->d_rp, g->d_col, g->d_perm, g->V, flag);
-        note_launch(1);
-        unsigned h = 0;
-        e = cudaMemcpy(&h, flag, 4, cudaMemcpyDeviceToHost);
-        if (e != cudaSuccess) return cuda_status(e, "overflow check");
-        if (h) return set_error(AG_ERR_OVERFLOW, "a finite distance exceeds 0xFFFFFFFE");
-    }
-    return AG_OK;
+    return set_error(AG_ERR_OVERFLOW, "a finite distance exceeds 0xFFFFFFFE");
 }
 
 static ag_status query(ag_graph g, int alg, uint32_t src, uint32_t *out, uint32_t *parents, const ag_policy *p,

@@ -120,6 +120,13 @@ struct alignas(128) Ctl {
     // others [leaders, nblocks); counters double-buffered by launch parity (the other half is zeroed)
     unsigned int sm_rank[256];        // CTAs that have arrived on SM s (mod CTAs per SM = rank on s)
     unsigned int lead_cnt[2], other_cnt[2];
+    // launches completed on this control block: its parity selects the (lead_cnt, other_cnt) pair of
+    // the next launch, which zeroes the other pair for the one after.  Advanced by the kernel itself
+    // (never by the host), so a call that fails before or at launch cannot desynchronise it.
+    unsigned int launch_seq;
+    // deferred status, sticky across launches until ag_graph_check() clears it: bit 0 = a finite
+    // distance exceeds MAX_FINITE (exact, checked in-kernel), bits 8.. = max abort code seen
+    unsigned int sticky;
 };
 
 // Policy as seen by the device (plain integers; filled from ag_policy on the host).

@@ -75,6 +75,7 @@ struct ag_local_group;
 
 struct ag_comm_s {
     int rank = 0, world = 1, device = 0;
+    int live_parts = 0;                // graphs partitioned over this comm and not yet freed
     ncclComm_t nccl = nullptr;
     ag_local_group *group = nullptr;   // virtual mode
 };
@@ -87,6 +88,7 @@ struct ag_local_group {
 
 struct ag_dist_part {
     ag_comm_s *comm = nullptr;
+    int world = 1;                     // copy of comm->world (the release path must not need the comm)
     uint32_t own_b = 0, own_e = 0;     // owned vertex range
     uint32_t S = 0;                    // slice size (bits), multiple of 1024
     uint32_t gwords = 0;               // words of the padded global bitmap (world * S / 32)
@@ -113,7 +115,8 @@ void dist_graph_release(ag_graph_s *g) {
     dev_free(d->d_next, (size_t)d->gwords * 4 + 128, g->device);
     dev_free(d->d_cnt, 64, g->device);
     if (d->h_cnt) cudaFreeHost(d->h_cnt);
-    const int W = d->comm ? d->comm->world : 1;
+    const int W = d->world;
+    if (d->comm) d->comm->live_parts -= 1;
     dev_free(d->d_send, (size_t)d->S * 8 + 128, g->device);
     dev_free(d->d_list, (size_t)W * d->S * 8 + 128, g->device);
     dev_free(d->d_counts, (size_t)W * CW * 4 + 128, g->device);
@@ -350,6 +353,8 @@ namespace {
 ag_status part_alloc(ag_graph_s *g, ag_comm_s *c) {
     ag_dist_part *d = new ag_dist_part();
     d->comm = c;
+    d->world = c->world;
+    c->live_parts += 1;
     ag_dist_owned_range(g->V, c->rank, c->world, &d->own_b, &d->own_e);
     uint64_t S = ((uint64_t)g->V + c->world - 1) / c->world;
     S = (S + 1023) & ~1023ull;
@@ -407,7 +412,6 @@ ag_status launch_level(ag_graph_s *g, uint32_t L, uint32_t *parent_local, cudaSt
     a.hub = g->d_hub;
     a.hub_cap = g->hub_cap;
     a.ctl = (Ctl *)g->d_ctl;
-    a.epoch = ++g->epoch;
     a.has_hubs = g->info.max_deg >= HUB_DEG;
     auto fn = dist_level_kernel<Off>;
     int occ = 0;
@@ -463,7 +467,6 @@ ag_status launch_sssp_round(ag_graph_s *g, const uint2 *list, uint32_t n, uint32
     a.hub = g->d_hub;
     a.hub_cap = g->hub_cap;
     a.ctl = (Ctl *)g->d_ctl;
-    a.epoch = ++g->epoch;
     a.has_hubs = g->info.max_deg >= HUB_DEG;
     a.ulist = list;
     auto fn = dist_sssp_kernel<Off>;
@@ -568,6 +571,9 @@ ag_status ag_dist_init_local(int world, int device, ag_comm *comms_out) {
 
 ag_status ag_dist_free(ag_comm c) {
     if (!c) return set_error(AG_ERR_INVALID_ARG, "NULL");
+    if (c->live_parts > 0)
+        return set_error(AG_ERR_INVALID_ARG, "ag_dist_free: %d graph(s) partitioned over this comm are still live; "
+                         "ag_graph_free them first", c->live_parts);
     if (c->nccl && g_nccl.ok) g_nccl.CommDestroy(c->nccl);
     if (c->group) {
         c->group->parts[c->rank] = nullptr;

@@ -55,11 +55,8 @@ struct ag_graph_s {
     size_t persist_bytes = 0;      // L2 persisting set-aside available
     size_t max_window = 0;         // cudaDeviceProp::accessPolicyMaxWindowSize
     cudaEvent_t ev[2] = {nullptr, nullptr};
-    uint32_t epoch = 0;
-    // deferred status of the last enqueued traversal
+    // deferred status: stream of the last enqueued traversal (the status itself is Ctl::sticky)
     cudaStream_t last_stream = nullptr;
-    int last_alg = 0;
-    uint32_t *last_out = nullptr;
     bool pending_check = false;
     // multi-GPU
     ag_dist_part *dist = nullptr;

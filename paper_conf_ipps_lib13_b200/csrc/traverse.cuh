@@ -74,7 +74,6 @@ struct TravArgs {
     DevPolicy pol;
     uint32_t src;
     uint32_t nblocks;
-    uint32_t epoch;
     uint32_t max_iters;
     uint32_t has_hubs;
     const uint2 *ulist;         // listed working set (multi-GPU SSSP): entry i = (u, dist of u); the value
@@ -1048,21 +1047,24 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     // small-frontier mode: wake events seen so far (read before the barrier: no wake can precede it),
     // and the virtual CTA id: one leader per SM first, so a small iteration runs on every SM
     uint32_t wgen = ld_relaxed(&ctl->wake_gen);
-    const uint32_t lpar = a.epoch & 1u;
     if (threadIdx.x == 0) {
+        // launch parity from the device-side launch counter (advanced at the end of every launch,
+        // after this read: every CTA reads it before its first grid-barrier arrival)
+        const uint32_t lpar = ld_relaxed(&ctl->launch_seq) & 1u;
         uint32_t smid;
         asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
         const uint32_t per_sm = a.pol.small_ctas ? (a.nblocks + a.pol.small_ctas - 1) / a.pol.small_ctas : 1u;
         const bool leader = atomicAdd(&ctl->sm_rank[smid & 255u], 1u) % per_sm == 0u;
         sm.red32[1][0] = leader;
         sm.red32[1][1] = leader ? atomicAdd(&ctl->lead_cnt[lpar], 1u) : atomicAdd(&ctl->other_cnt[lpar], 1u);
+        sm.red32[1][2] = lpar;
         if (blockIdx.x == 0) {
             ctl->lead_cnt[lpar ^ 1u] = 0u;   // for the next launch (stream-ordered after this one)
             ctl->other_cnt[lpar ^ 1u] = 0u;
         }
     }
     grid_barrier(ctl, a.nblocks);
-    const uint32_t nlead = ld_relaxed(&ctl->lead_cnt[lpar]);
+    const uint32_t nlead = ld_relaxed(&ctl->lead_cnt[sm.red32[1][2]]);
     const uint32_t vid = sm.red32[1][0] ? sm.red32[1][1] : nlead + sm.red32[1][1];   // permutation of [0, nblocks)
     const uint32_t vgtid = vid * BS + threadIdx.x;
     __syncthreads();   // (red32 reuse)
@@ -1282,6 +1284,21 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         if (it > 0 && it - 1 < a.trace_cap && a.trace_edges) a.trace_edges[it - 1] = ld_relaxed64(&ctl->it_edges[(it + 2) % 3]);
         if (it >= a.max_iters) ctl->aborted = 1;
         if (it <= a.trace_cap && a.trace_ns) a.trace_ns[it] = globaltimer_ns();
+        const uint32_t ab = ld_relaxed(&ctl->aborted);
+        if (ab) atomicMax(&ctl->sticky, ab << 8);
+        ctl->launch_seq += 1u;   // every CTA read it before the first grid barrier
+    }
+    // exact overflow test (rare path: only when a relaxation exceeded MAX_FINITE): a reachable vertex
+    // left at INF behind a finite one.  The packed state is final here (every CTA passed the barrier
+    // that ended the last iteration, or was parked without writing), so no further barrier is needed.
+    if (ALG == ALG_SSSP && !a.ulist && ld_relaxed(&ctl->overflow)) {
+        bool bad = false;
+        for (uint32_t u = gtid; u < a.V && !bad; u += gthreads) {
+            if ((a.P[u] >> 32) == INF) continue;
+            for (Off e = a.rp[u]; e < a.rp[u + 1]; ++e)
+                if ((a.P[a.cw[e].x] >> 32) == INF) { bad = true; break; }
+        }
+        if (bad) atomicOr(&ctl->sticky, 1u);
     }
     if (ALG == ALG_SSSP) {  // unpack (dist, parent) into the caller's arrays (caller ids)
         for (uint32_t v = gtid; v < a.V; v += gthreads) {

@@ -74,8 +74,8 @@ def check_bfs(g, G, s, p, expect_level=None, want_parents=True):
     return st
 
 
-def check_sssp(g, G, s, p):
-    d, _ = oracle.dijkstra(g, s)
+def check_sssp(g, G, s, p, expect_dist=None):
+    d = oracle.dijkstra(g, s, want_parents=False)[0] if expect_dist is None else expect_dist
     parents = np.empty(g.V, np.uint32)
     out, _, st = G.sssp(s, parents=parents, policy=p, stats=True)
     assert np.array_equal(out, d), f"SSSP dist differ ({pname(p)}, src {s}): {np.count_nonzero(out != d)} mismatches"
@@ -449,3 +449,45 @@ def test_allocator_hook_switched_between_load_and_free():
         A.use_torch_allocator(False)
         sys.unraisablehook = old
     assert not errs, errs
+
+
+def test_failed_call_does_not_desynchronise_launch_parity():
+    """A call rejected before launch (ordered CC) must not break the next traversals on the handle:
+    the small-frontier mode's virtual-CTA counters are double-buffered by a DEVICE launch counter,
+    so the host can never consume a parity without a launch."""
+    g = aggen.config("C1")
+    G = A.Graph.from_csr(g)
+    lab = oracle.cc(g)
+    s = int(aggen.sources(g, 1)[0])
+    lv, _ = oracle.bfs(g, s, want_parents=False)
+    assert np.array_equal(G.cc()[0], lab)
+    for _ in range(3):
+        with pytest.raises(A.AgError) as e:
+            G.cc(policy=pol(1))
+        assert e.value.status == "AG_ERR_UNSUPPORTED"
+        assert np.array_equal(G.cc()[0], lab)
+        assert np.array_equal(G.bfs(s)[0], lv)
+
+
+def test_deferred_overflow_is_sticky_across_queries():
+    """An overflow of an EARLIER enqueued SSSP is still reported by ag_graph_check after later
+    queries on the same handle were enqueued, and the check clears it."""
+    import torch
+    g = aggen.path(4)
+    g.w = np.full(g.E, 0x7FFFFFFF, np.uint32)     # 0 -> 3 is 3 * (2^31 - 1) > 0xFFFFFFFE
+    G = A.Graph.from_csr(g)
+    out = torch.empty(g.V, dtype=torch.int32, device="cuda")
+    stream = torch.cuda.current_stream().cuda_stream
+    G.sssp(0, dist=out, stream=stream)             # overflows
+    G.sssp(3, dist=out, stream=stream)             # from the other end: also overflows
+    G.sssp(1, dist=out, stream=stream)             # 1 -> 3 = 2 * (2^31 - 1) = 0xFFFFFFFE: fine
+    with pytest.raises(A.AgError) as e:
+        G.check()
+    assert e.value.status == "AG_ERR_OVERFLOW"
+    G.check()                                      # cleared
+    assert list(out.cpu().numpy().view(np.uint32)) == [0x7FFFFFFF, 0, 0x7FFFFFFF, 0xFFFFFFFE]
+    G.sssp(0, dist=out, stream=stream)
+    G.sssp(1, dist=out, stream=stream)
+    with pytest.raises(A.AgError) as e:           # the earlier overflow survives the later good query
+        G.check()
+    assert e.value.status == "AG_ERR_OVERFLOW"

@@ -170,6 +170,7 @@ def test_invariants_and_symmetry_c1():
     g = aggen.config("C1")
     srcs = aggen.sources(g, 3)
     comp = bf.components(g)
+    comp_e = bf.component_edge_entries(g)
     D = {}
     for s in srcs:
         dist, par = oracle.dijkstra(g, s)
@@ -178,7 +179,7 @@ def test_invariants_and_symmetry_c1():
         assert oracle.validate(g, s, level, lpar)[0] == 0
         Vr, Er = oracle.reached(g, dist)
         assert Vr == comp[s]                       # union-find component size
-        assert Er == int(np.diff(g.row_ptr)[dist != INF].sum())
+        assert Er == comp_e[s]                     # edge-list entries leaving s's union-find component
         assert np.array_equal(level != INF, dist != INF)
         D[int(s)] = dist.astype(np.int64)
     a, b, c = [int(x) for x in srcs]
@@ -200,6 +201,24 @@ def test_validator_rejects_corruption():
     assert oracle.validate(g, s, dist, bp, weighted=True)[0] in (3, 4)
     bad = dist.copy(); bad[s] = 1
     assert oracle.validate(g, s, bad, par, weighted=True)[0] == 1
+
+
+def test_validator_rejects_parent_corruption_codes_5_and_6():
+    """Certificate rule 4: an unreached vertex must have parent INF (code 5) and the
+    source must be its own parent (code 6, Graph500 convention) — each corruption alone is rejected
+    with its own code, and the uncorrupted certificate passes."""
+    g = aggen.csr_from_edges(6, [0, 1, 1, 3], [1, 0, 2, 4], w=[2, 2, 5, 1])   # 3 -> 4 and 5 unreachable from 0
+    for weighted in (False, True):
+        out, par = (oracle.dijkstra(g, 0) if weighted else oracle.bfs(g, 0))
+        assert list(out[[3, 4, 5]]) == [INF] * 3 and oracle.validate(g, 0, out, par, weighted)[0] == 0
+        bp = par.copy(); bp[4] = 3                    # unreached vertex 4 claims the real edge (3, 4)
+        assert oracle.validate(g, 0, out, bp, weighted) == (5, 4)
+        bp = par.copy(); bp[5] = 0
+        assert oracle.validate(g, 0, out, bp, weighted) == (5, 5)
+        bp = par.copy(); bp[0] = 1                    # the source's parent is not itself
+        assert oracle.validate(g, 0, out, bp, weighted) == (6, 0)
+        bp = par.copy(); bp[0] = INF
+        assert oracle.validate(g, 0, out, bp, weighted) == (6, 0)
 
 
 def test_bfs_level_sizes_definition():

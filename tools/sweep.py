@@ -6,6 +6,10 @@
 For each variant (order x mapping x workset, plus the paper and tuned adaptive policies) prints the
 median device time over the sources, GTEPS (E_r / t), iterations and optionally the per-iteration
 trace (|WS|, edges, variant, microseconds).  Device times come from the library's CUDA events.
+
+--expect FILE (written by `python -m tests.oracle_expect`, the oracle's levels / distances for the
+same seeded sources): every run's output is compared element by element before its time is kept;
+a mismatch is recorded as {"verified": false, ...} with no time.  Rows carry "verified": true.
 """
 import argparse
 import json
@@ -47,7 +51,9 @@ def main():
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--delta", type=int, default=1)
     ap.add_argument("--set", default="", help="extra policy fields k=v,k=v")
+    ap.add_argument("--expect", default="", help="oracle results (.npz from tests/oracle_expect.py)")
     args = ap.parse_args()
+    expect = np.load(args.expect) if args.expect else None
     g = aggen.config(args.config)
     G = A.Graph.from_csr(g)
     srcs = [int(s) for s in aggen.sources(g, args.sources, seed=3)]
@@ -67,12 +73,15 @@ def main():
             for k, v in extra.items():
                 setattr(p, k, int(v))
             times, edges, iters, traces, red = [], [], [], [], []
+            bad = None
             try:
                 for s in srcs:
                     best = None
                     for _ in range(args.reps):
                         fn = G.bfs if alg == "bfs" else G.sssp
-                        _, _, st = fn(s, policy=p, stats=True, trace_cap=1 << 20 if args.trace else 0)
+                        out, _, st = fn(s, policy=p, stats=True, trace_cap=1 << 20 if args.trace else 0)
+                        if expect is not None and not np.array_equal(out, expect[f"{alg}_{s}"]):
+                            bad = (s, int(np.count_nonzero(out != expect[f"{alg}_{s}"])))
                         if best is None or st.device_ms < best.device_ms:
                             best = st
                     times.append(best.device_ms)
@@ -86,7 +95,11 @@ def main():
             except A.AgError as e:
                 print(json.dumps({"alg": alg, "variant": name, "error": str(e)}), flush=True)
                 continue
-            rec = {"alg": alg, "variant": name, "ms_median": statistics.median(times),
+            if bad is not None:
+                print(json.dumps({"alg": alg, "variant": name, "verified": False, "source": bad[0],
+                                  "mismatches": bad[1]}), flush=True)
+                continue
+            rec = {"alg": alg, "variant": name, "verified": expect is not None, "ms_median": statistics.median(times),
                    "gteps": sum(edges) / (sum(times) * 1e-3) / 1e9, "iters": statistics.median(iters),
                    "redundancy": round(statistics.median(red), 3),
                    "ms_all": [round(t, 3) for t in times]}
