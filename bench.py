@@ -119,6 +119,19 @@ def load_traffic(cfg):
         return None
 
 
+def cpu_model():
+    """The host CPU model (from /proc/cpuinfo) and the number of online cores."""
+    name = "unknown"
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                name = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"model": name, "online_cores": os.cpu_count()}
+
+
 def run_reference(args, rank, world):
     """The oracle as it stands, on this host's cores (rank 0 only)."""
     if rank != 0:
@@ -155,7 +168,8 @@ def run_reference(args, rank, world):
            "dtype": "u32", "data": "synthetic",
            "config": {"workload": f"{args.config}: {CONFIG_DESC.get(args.config, '')}; BFS + SSSP per step",
                       "V": g.V, "E": g.E},
-           "cpu_baseline": {"value": val, "unit": "GTEPS", "cores": 1, "kind": "oracle", "sample": sample},
+           "cpu_baseline": {"value": val, "unit": "GTEPS", "cores": 1, "kind": "oracle", "sample": sample,
+                            "cpu": cpu_model()},
            "e2e": {"value": val, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
 
@@ -172,8 +186,45 @@ def cpu_baseline(g, srcs, budget_s=20.0):
         n += 1
         if t > budget_s:
             break
-    return {"value": e / t / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+    return {"value": e / t / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle", "cpu": cpu_model(),
             "sample": f"{n} sources x (queue BFS + heap Dijkstra) on the full graph, serial, {t:.1f}s"}
+
+
+def side_configs(A, aggen, local, reps=3):
+    """The other single-GPU configs of BASELINE.json (C3 grid: ordered vs unordered SSSP; C4 ER: the
+    bitmap vs queue crossover), timed with the library's own CUDA events on the adaptive tuned policy —
+    reported beside the C2 step, not part of it.  For the latency-bound grid also the floor
+    D x t_iter_min: levels x the fastest single iteration of the same traversal."""
+    out = {}
+    for cfg in ("C3", "C4"):
+        g = aggen.config(cfg)
+        G = A.Graph.from_csr(g, device=local)
+        s = int(aggen.sources(g, 1, seed=3)[0])
+        rec = {"V": g.V, "E": g.E, "source": s}
+        for name, fn, order in (("bfs", G.bfs, 0), ("sssp", G.sssp, 0), ("sssp_ordered", G.sssp, 1)):
+            p = A.policy_default(local)
+            p.order = order
+            if cfg == "C3" and order == 1:
+                p.delta = 64
+            best = None
+            for _ in range(reps):
+                _, _, st = fn(s, policy=p, stats=True, trace_cap=1 << 16)
+                if best is None or st.device_ms < best.device_ms:
+                    best = st
+            r = {"ms": round(best.device_ms, 3), "gteps": best.reached_edges / (best.device_ms * 1e-3) / 1e9,
+                 "iterations": best.iterations}
+            if order == 1:
+                r["delta"] = int(p.delta)
+            us = getattr(best, "trace_us", None)
+            if cfg == "C3" and us is not None and len(us):
+                tmin = float(np.min(us))
+                r["t_iter_min_us"] = round(tmin, 2)
+                r["latency_floor_ms"] = round(best.iterations * tmin / 1e3, 3)
+                r["floor_frac"] = round(best.iterations * tmin / 1e3 / best.device_ms, 3)
+            rec[name] = r
+        out[cfg] = rec
+        G.free()
+    return out
 
 
 def run_dist(args, rank, world, local, dist):
@@ -317,6 +368,7 @@ def main():
     ap.add_argument("--config", default="C2")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-extra", action="store_true", help="skip the C3/C4 side measurements")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -460,6 +512,9 @@ def main():
     tc = statistics.median(evc[k].elapsed_time(evc[k + 1]) for k in range(kc))
     out["cc"] = {"ms": tc, "gteps": g.E / (tc * 1e-3) / 1e9, "iterations": sc.iterations,
                  "edges_inspected_per_E": sc.edges_inspected / max(1, g.E), "runs": kc}
+
+    if not args.no_extra and world == 1:
+        out["other_configs"] = side_configs(A, aggen, local)
 
     # end-to-end through the public API with HOST buffers: CSR upload from pinned memory, both
     # traversals, results read back (the paper's timing scope, 26.s17-18; reading R21)

@@ -35,6 +35,7 @@ extern "C" {
 #define AG_ABI_VERSION 1u
 #define AG_INF 0xFFFFFFFFu
 #define AG_WINDOW_AUTO 0xFFFFFFFFu
+#define AG_WINDOW_ADAPTIVE 0xFFFFFFFEu   /* sssp_window: adapted per iteration (NEXT-3) */
 
 typedef struct ag_graph_s *ag_graph; /* opaque, library-owned device CSR + scratch */
 typedef struct ag_comm_s *ag_comm;   /* opaque multi-GPU communicator (one per process/GPU) */
@@ -84,12 +85,16 @@ typedef struct {
     uint64_t t2_ws;          /* T2, default thread_tpb x #SMs (28.s24-27; reading R17) */
     uint32_t t3_ppm;         /* T3 = ceil(t3_ppm * V / 1e6) (Fig. 13 sweeps 1-13% of V; reading R14) */
     uint32_t sample_every;   /* inspector sampling interval (26.s7-9; reading R15), >= 1 */
-    uint32_t delta;          /* ordered-SSSP bucket width; 1 = the paper's Dijkstra batches (28.s8, R9) */
+    uint32_t delta;          /* ordered-SSSP bucket width; 1 = the paper's Dijkstra batches (28.s8, R9);
+                                0 = adaptive (NEXT-3): starts at 1 and is halved / doubled every iteration
+                                from the measured re-expansion ratio (> 1/4: halve, < 1/16: double) */
     uint32_t thread_tpb;     /* thread-mapping block size used for T2, paper 192 (26.s27) */
     uint32_t cta_group;      /* block-mapping group size (multiple of 32); 0 = auto (26.s28, R16) */
     uint32_t sssp_window;    /* unordered SSSP: expand only frontier vertices with dist < min + window
                                 (others stay in the working set); 0 = off (plain Bellman-Ford rounds);
-                                AG_WINDOW_AUTO = tuned: off on skewed graphs, else 8 x max_weight / avg degree */
+                                AG_WINDOW_AUTO = tuned: off on skewed graphs, else 8 x max_weight / avg degree;
+                                AG_WINDOW_ADAPTIVE = NEXT-3: start at that value, then halve / double it every
+                                iteration from the measured re-expansion ratio (the order axis at run time) */
     uint32_t sssp_hub_window;/* unordered SSSP: vertices with out-degree >= 64 are expanded only when within
                                 this distance of the frontier minimum (re-expanding a hub re-scans its whole
                                 list); 0 = off; AG_WINDOW_AUTO = tuned: max(1, max_weight / 50) */
@@ -102,7 +107,9 @@ typedef struct {
                                 skewed graphs: a diagnostic / test setting).  BFS and ag_cc use t_free from this
                                 field, ag_sssp the same threshold.
                                 0 = never; ag_policy_default: 3906 (V/256) */
-    uint32_t reserved;       /* must be 0 */
+    uint32_t small_ws;       /* tuned policy, graphs without hub lists: an iteration whose working set has fewer than
+                                small_ws elements runs on one CTA per SM while the others park (cheaper grid barrier;
+                                DESIGN.md §5); 0 = AUTO (32768); 0xFFFFFFFF = always; 1 = never.  Results unchanged. */
 } ag_policy;
 
 typedef struct {

@@ -24,6 +24,7 @@ WS_AUTO, WS_BITMAP, WS_QUEUE = 0, 1, 2
 POLICY_PAPER, POLICY_TUNED = 0, 1
 LAYOUT_AUTO, LAYOUT_IDENTITY, LAYOUT_DEGREE = 0, 1, 2
 WINDOW_AUTO = 0xFFFFFFFF
+WINDOW_ADAPTIVE = 0xFFFFFFFE
 STATUS = {0: "AG_OK", 1: "AG_ERR_INVALID_ARG", 2: "AG_ERR_BAD_CSR", 3: "AG_ERR_SRC_RANGE", 4: "AG_ERR_NO_WEIGHTS",
           5: "AG_ERR_OVERFLOW", 6: "AG_ERR_OOM", 7: "AG_ERR_CUDA", 8: "AG_ERR_NCCL", 9: "AG_ERR_UNSUPPORTED",
           10: "AG_ERR_NO_DEVICE"}
@@ -52,7 +53,7 @@ class Policy(ctypes.Structure):
                 ("t2_ws", ctypes.c_uint64), ("t3_ppm", ctypes.c_uint32), ("sample_every", ctypes.c_uint32),
                 ("delta", ctypes.c_uint32), ("thread_tpb", ctypes.c_uint32), ("cta_group", ctypes.c_uint32),
                 ("sssp_window", ctypes.c_uint32), ("sssp_hub_window", ctypes.c_uint32), ("free_ppm", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32)]
+                ("small_ws", ctypes.c_uint32)]
 
 
 class GraphInfo(ctypes.Structure):

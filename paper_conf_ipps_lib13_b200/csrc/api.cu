@@ -264,6 +264,21 @@ __global__ void reached_kernel(const uint32_t *out, const Off *rp, const uint32_
     if ((threadIdx.x & 31) == 0 && (a | b)) { atomicAdd(&acc[0], a); atomicAdd(&acc[1], b); }
 }
 
+// Exact overflow test after an SSSP traversal (enqueued behind it; returns at once unless a relaxation
+// exceeded MAX_FINITE): a reachable vertex left at INF behind a finite one.  Packed state in device ids.
+template <typename Off>
+__global__ void overflow_check_kernel(const Ctl *ctl, const unsigned long long *P, const Off *rp, const uint2 *cw, uint32_t V,
+                                      unsigned *sticky) {
+    if (!*(volatile const unsigned *)&ctl->overflow) return;
+    bool bad = false;
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < V && !bad; u += gridDim.x * blockDim.x) {
+        if ((P[u] >> 32) == INF) continue;
+        for (Off e = rp[u]; e < rp[u + 1]; ++e)
+            if ((P[cw[e].x] >> 32) == INF) { bad = true; break; }
+    }
+    if (bad) atomicOr(sticky, 1u);
+}
+
 // ------------------------------------------------------------------------------------------------
 // graph handle helpers
 // ------------------------------------------------------------------------------------------------
@@ -315,7 +330,7 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
     d.t2 = p.t2_ws;
     d.t3 = ((uint64_t)g.V * p.t3_ppm + 999999ull) / 1000000ull;
     d.sample_every = p.sample_every ? p.sample_every : 1;
-    d.delta = p.delta ? p.delta : 1;
+    d.delta = p.delta ? p.delta : 1;   // 0 = adaptive, starting at 1 (below)
     uint32_t grp = p.cta_group;
     if (grp == 0) {  // multiple of 32 closest to the average out-degree, ties up (26.s28, R16)
         uint64_t k = g.V ? (2 * g.E + 32ull * g.V) / (64ull * g.V) : 1;
@@ -325,7 +340,7 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
     grp = grp > (uint32_t)BS ? (uint32_t)BS : grp;
     grp &= ~31u;
     d.cta_group = grp;
-    if (p.sssp_window == AG_WINDOW_AUTO) {
+    if (p.sssp_window == AG_WINDOW_AUTO || p.sssp_window == AG_WINDOW_ADAPTIVE) {
         // tuned: Bellman-Ford re-expansion is distance-ordering waste on long-path graphs (grid: 152x,
         // ER: 4.3x) but not on power-law graphs (R-MAT: no gain) -- measured with tools/sweep.py
         const uint64_t avg = g.V ? (g.E + g.V - 1) / g.V : 1;
@@ -334,6 +349,7 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
         if (w < 1) w = 1;
         if (w > 0x7FFFFFFFull) w = 0x7FFFFFFFull;
         d.window = (p.kind == AG_POLICY_TUNED && !skewed && g.info.max_weight) ? (uint32_t)w : 0u;
+        if (p.sssp_window == AG_WINDOW_ADAPTIVE) d.window = (uint32_t)w;   // the start of the adapted window
     } else {
         d.window = p.sssp_window;
     }
@@ -365,12 +381,13 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
     // on one CTA per SM, the others park — the grid barrier that ends every iteration then has 148
     // arrivals instead of ~740 (measured C3 grid: BFS 55.9 -> 42.4 ms, SSSP 129 -> 92.7 ms with 148 CTAs)
     d.small_ctas = (uint32_t)g.num_sms;
-    d.t_small = p.kind == AG_POLICY_TUNED ? 32768u : 0u;
-    if (const char *ts = getenv("AG_SMALL_WS")) d.t_small = (uint32_t)atoi(ts);   // experiments / tests
+    d.t_small = p.kind == AG_POLICY_TUNED ? (p.small_ws ? p.small_ws : 32768u) : 0u;
     d.t_small_hub = p.kind == AG_POLICY_TUNED ? 4096u : 0u;   // C2: BFS -1.6%, SSSP -2.7% (median of 12)
-    if (const char *ts = getenv("AG_SMALL_HUB_WS")) d.t_small_hub = (uint32_t)atoi(ts);
     d.smallchunk_per_cta = SMALLCHUNK_PER_CTA;
-    if (const char *ts = getenv("AG_SMALLCHUNK_PER_CTA")) d.smallchunk_per_cta = (uint32_t)atoi(ts);   // experiments
+    d.ordered = p.order == AG_ORDERED ? 1u : 0u;
+    // NEXT-3: the SSSP order axis adapted per iteration from the measured redundancy
+    d.adapt = (p.order == AG_ORDERED) ? (p.delta == 0 ? 1u : 0u) : (p.sssp_window == AG_WINDOW_ADAPTIVE ? 1u : 0u);
+    d.win_max = 1u << 24;
     return d;
 }
 
@@ -379,7 +396,7 @@ ag_status check_policy(const ag_policy *p) {
     if (p->order > AG_ORDERED || p->mapping > AG_MAP_HYBRID || p->workset > AG_WS_QUEUE || p->kind > AG_POLICY_TUNED)
         return set_error(AG_ERR_INVALID_ARG, "ag_policy field out of range");
     if (p->cta_group % 32) return set_error(AG_ERR_INVALID_ARG, "cta_group must be a multiple of 32");
-    if (p->delta == 0 || p->delta >= 0x80000000u) return set_error(AG_ERR_INVALID_ARG, "delta must be in [1, 2^31)");
+    if (p->delta >= 0x80000000u) return set_error(AG_ERR_INVALID_ARG, "delta must be 0 (adaptive) or in [1, 2^31)");
     return AG_OK;
 }
 
@@ -404,16 +421,13 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
     if (e != cudaSuccess || occ < 1) return cuda_status(e == cudaSuccess ? cudaErrorLaunchOutOfResources : e, "occupancy");
     // L1/shared carveout: request just the shared memory the resident CTAs need so the rest of the
     // 256 KB goes to L1, where the status gathers hit (the driver otherwise picked a 132 KB shared
-    // configuration for ~100 KB of use).  Once per kernel; AG_CARVEOUT=<pct> or -1 overrides.
+    // configuration for ~100 KB of use).  Once per kernel.
     static int carved[2] = {0, 0};   // per specialisation (tuned / paper variants)
     if (!carved[tuned]) {
         carved[tuned] = 1;
         int pct = -1;
-        const char *ev = getenv("AG_CARVEOUT");
         cudaFuncAttributes fa;
-        if (ev) {
-            pct = atoi(ev);
-        } else if (cudaFuncGetAttributes(&fa, fn) == cudaSuccess) {
+        if (cudaFuncGetAttributes(&fa, fn) == cudaSuccess) {
             const double need = (double)occ * ((double)fa.sharedSizeBytes + dyn + 1024.0);
             pct = (int)((need * 100.0 + 228.0 * 1024.0 - 1.0) / (228.0 * 1024.0));
             if (pct > 100) pct = 100;
@@ -428,10 +442,6 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
         cudaGetLastError();
     }
     a.nblocks = (uint32_t)(occ * g->num_sms);
-    if (const char *nb = getenv("AG_NBLOCKS")) {   // experiment knob: cap the persistent grid
-        const uint32_t cap = (uint32_t)atoi(nb);
-        if (cap >= 1 && cap < a.nblocks) a.nblocks = cap;
-    }
     // Cooperative launch (co-resident grid for the software grid barrier) with an L2 access-policy
     // window marking the per-vertex status array persisting, so the ~1 GB CSR stream does not evict
     // it.  The window is a per-launch attribute: the caller's stream is not modified.
@@ -446,7 +456,7 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
     int nattr = 1;
     void *wbase = ALG == ALG_SSSP ? (void *)a.P : ALG == ALG_CC ? (void *)a.level : (void *)a.vis;
     size_t wbytes = ALG == ALG_SSSP ? (size_t)g->V * 8 : ALG == ALG_CC ? (size_t)g->V * 4 : (size_t)g->nwords * 4;
-    if (g->persist_bytes > 0 && getenv("AG_NO_L2_WINDOW") == nullptr) {
+    if (g->persist_bytes > 0) {
         if (wbytes > g->max_window) wbytes = g->max_window;
         attrs[1].id = cudaLaunchAttributeAccessPolicyWindow;
         attrs[1].val.accessPolicyWindow.base_ptr = wbase;
@@ -563,6 +573,12 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
     }
     if (s != AG_OK) return s;
     if (stats) cudaEventRecord(g->ev[1], st);
+    if (alg == ALG_SSSP) {   // deferred exact overflow test (a no-op launch unless the traversal flagged one)
+        Ctl *ctl = (Ctl *)g->d_ctl;
+        overflow_check_kernel<Off><<<g->num_sms * 4, 256, 0, st>>>(ctl, g->d_P, (const Off *)g->d_rp, g->d_cw, g->V,
+                                                                    &ctl->sticky);
+        note_launch(1);
+    }
     g->last_stream = st;
     g->pending_check = true;
 

@@ -103,7 +103,9 @@ struct alignas(128) Ctl {
     unsigned int hub_tail[3];         // hybrid mapping: produced hub-chunk tasks
     unsigned int hub_head[3];         //                 consumed hub-chunk tasks
     unsigned int stage_done[3];       //                 CTAs done producing
-    unsigned long long it_edges[3];   // edges inspected in iteration (trace only)
+    unsigned long long it_edges[3];   // edges inspected in iteration (m_F: selector input, trace)
+    unsigned long long it_nv[3];      // working-set elements expanded in iteration
+    unsigned int it_reexp[3];         // SSSP: expansions of a vertex already expanded earlier in the query
     unsigned int free_any[3];         // free-output iteration wrote at least one next-bitmap bit
     unsigned int pend_count;          // ordered SSSP: |pending|
     unsigned int overflow;            // a relaxation exceeded MAX_FINITE
@@ -115,7 +117,8 @@ struct alignas(128) Ctl {
     // it, and must not slow the atomics on the per-iteration counters above.
     alignas(128) unsigned int wake_gen;   // wake events so far (monotone across launches)
     unsigned int wake_it, wake_n, wake_nprev;
-    unsigned int pad2[28];
+    unsigned int wake_win;            //   ... and the current adaptive window / bucket width
+    unsigned int pad2[27];
     // virtual CTA numbering (small-frontier mode): one "leader" CTA per SM gets vid [0, leaders), the
     // others [leaders, nblocks); counters double-buffered by launch parity (the other half is zeroed)
     unsigned int sm_rank[256];        // CTAs that have arrived on SM s (mod CTAs per SM = rank on s)
@@ -152,17 +155,24 @@ struct DevPolicy {
     uint32_t t_small;     //   0 = off
     uint32_t t_small_hub; //   graphs with hub tasks: only in the shrinking tail (|WS| below this and falling)
     uint32_t smallchunk_per_cta;  // tuned kernels: |WS| < this x CTAs -> HUB_CHUNK_SMALL-entry hub tasks
+    uint32_t ordered;     // ordered SSSP: |WS| is the pending set (its representation is selected)
+    uint32_t adapt;       // SSSP order axis adapted per iteration (NEXT-3): the unordered deferral window
+                          // (sssp_window = AG_WINDOW_ADAPTIVE) or the ordered bucket width (delta = 0)
+    uint32_t win_max;     //   upper bound of the adapted window / width
 };
 
 // The decision maker.  PAPER: Fig. 11 with readings R12/R13:
 //   ws < T2 -> B_QU; else workset = ws >= T3 ? BM : QU; mapping = E >= T1*V ? B : T.
-// TUNED (B200, calibrated by tools/sweep.py on C2/C3/C4): the queue always wins on
-//   B200 (appends are warp-aggregated, the bitmap scan is O(V) threads per iteration); mapping is
-//   THREAD for small working sets of a graph whose max out-degree is <= 64 (no straggler risk, no
-//   tile-scan overhead), else HYBRID (load-balanced gather + hub splitting).
+// TUNED (B200, calibrated with tools/sweep.py / tools/calibrate.py on C2/C3/C4), from
+//   |WS| and m_F (the working set's out-degree sum; the kernel passes |WS| x the previous frontier's
+//   average degree, the paper's inspector statistic, 26.s4-7):
+//   * working set: the queue (appends are warp-staged, the bitmap scan costs O(V/32) per iteration),
+//     except the ordered-SSSP pending set once it holds >= V/32 vertices: a bucket then re-reads most
+//     of it, and one O(V/32) scan of the pending bitmap beats re-reading (and re-appending) the list;
+//   * mapping: THREAD for small working sets of low out-degree (m_F <= 16 |WS|) on graphs without
+//     straggler lists (max degree <= 64), else HYBRID (load-balanced pieces + hub tasks).
 __host__ __device__ inline uint8_t select_variant(const DevPolicy &p, uint64_t ws, uint64_t ws_edges) {
     uint32_t map, wsr;
-    (void)ws_edges;
     if (p.kind == AG_POLICY_PAPER) {
         if (ws < p.t2) {
             map = MAP_B;
@@ -172,8 +182,9 @@ __host__ __device__ inline uint8_t select_variant(const DevPolicy &p, uint64_t w
             map = (p.E >= (uint64_t)p.t1 * p.V) ? MAP_B : MAP_T;
         }
     } else {
-        wsr = WS_QU;
-        map = (p.max_deg <= 64 && ws < p.t2_tuned) ? MAP_T : MAP_H;
+        wsr = (p.ordered && ws >= ((uint64_t)p.V + 31) / 32) ? WS_BM : WS_QU;
+        const bool low_deg = ws_edges <= 16ull * ws;
+        map = (p.max_deg <= 64 && low_deg && ws < p.t2_tuned) ? MAP_T : MAP_H;
     }
     if (p.force_map) map = p.force_map;
     if (p.force_ws) wsr = p.force_ws;
@@ -286,8 +297,10 @@ __device__ __forceinline__ void mbar_wait(uint64_t *mbar, unsigned parity) {
     while (!mbar_try_wait(mbar, parity)) {
     }
 }
-// cp.async (LDGSTS) 16-byte global -> shared, L1 bypass, with an L2 policy
-__device__ __forceinline__ void cp_async16(void *dst, const void *src, uint64_t) {
+// cp.async (LDGSTS) 16-byte global -> shared, L1 bypass.  (The .L2::cache_hint form compiled to an
+// LDGSTS whose policy descriptor faulted with "illegal instruction" on B200 when issued from a second
+// call site of the same kernel — measured with compute-sanitizer, tools/star_repro.py — so no hint.)
+__device__ __forceinline__ void cp_async16(void *dst, const void *src) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }

@@ -96,6 +96,11 @@ struct ag_dist_part {
     uint32_t *d_next = nullptr;        // next-frontier bitmap (only owned words written)
     unsigned long long *d_cnt = nullptr;
     unsigned long long *h_cnt = nullptr;  // pinned
+    unsigned *d_done = nullptr;        // BFS device-side termination: [0] frontier empty, [1] block arrivals,
+                                       // [2] levels after the first, [3] |WS| of the next level
+    unsigned *h_done = nullptr;        // pinned copy, read once per batch of enqueued levels
+    uint32_t *d_trace = nullptr;       // per-level frontier sizes (stats)
+    uint32_t trace_cap = 0;
     // SSSP exchange buffers (allocated on the first ag_dist_sssp)
     uint2 *d_send = nullptr;           // S entries: (owned improved vertex, its distance)
     uint2 *d_list = nullptr;           // world * S entries: the gathered global frontier
@@ -115,6 +120,9 @@ void dist_graph_release(ag_graph_s *g) {
     dev_free(d->d_next, (size_t)d->gwords * 4 + 128, g->device);
     dev_free(d->d_cnt, 64, g->device);
     if (d->h_cnt) cudaFreeHost(d->h_cnt);
+    dev_free(d->d_done, 64, g->device);
+    if (d->h_done) cudaFreeHost(d->h_done);
+    dev_free(d->d_trace, (size_t)d->trace_cap * 4 + 64, g->device);
     const int W = d->world;
     if (d->comm) d->comm->live_parts -= 1;
     dev_free(d->d_send, (size_t)d->S * 8 + 128, g->device);
@@ -198,44 +206,97 @@ __global__ void owned_check_kernel(const uint32_t *col, uint64_t E, uint32_t b, 
         if (col[k] < b || col[k] >= e) *bad = 1;
 }
 
-__global__ void popcount_kernel(const uint32_t *bm, uint32_t nwords, unsigned long long *cnt) {
+// After the exchange of a level: clear this rank's owned next slice, count the gathered frontier (every
+// rank holds the same bitmap, so every rank takes the same decision), record |WS| of the next level
+// and set done[0] when it is empty.  The last block to finish decides.
+__global__ void dist_level_finish_kernel(const uint32_t *front, uint32_t gwords, uint32_t *next_owned, uint32_t owned_words,
+                                         unsigned long long *cnt, unsigned *done, uint32_t *trace, uint32_t trace_cap) {
+    __shared__ unsigned long long part[32];
     unsigned long long c = 0;
-    for (uint32_t wi = blockIdx.x * blockDim.x + threadIdx.x; wi < nwords; wi += gridDim.x * blockDim.x)
-        c += __popc(bm[wi]);
+    for (uint32_t wi = blockIdx.x * blockDim.x + threadIdx.x; wi < gwords; wi += gridDim.x * blockDim.x) c += __popc(front[wi]);
+    for (uint32_t wi = blockIdx.x * blockDim.x + threadIdx.x; wi < owned_words; wi += gridDim.x * blockDim.x) next_owned[wi] = 0u;
     c = warp_sum(c);
-    if ((threadIdx.x & 31) == 0 && c) atomicAdd(cnt, c);
+    if ((threadIdx.x & 31) == 0) part[threadIdx.x >> 5] = c;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long t = 0;
+        for (uint32_t i = 0; i < blockDim.x / 32; ++i) t += part[i];
+        if (t) atomicAdd(cnt, t);
+        __threadfence();
+        if (atomicAdd(done + 1, 1u) == gridDim.x - 1) {
+            __threadfence();
+            const unsigned long long tot = *(volatile unsigned long long *)cnt;
+            if (!*(volatile unsigned *)done) {
+                done[3] = (unsigned)(tot > 0xFFFFFFFFull ? 0xFFFFFFFFull : tot);
+                if (tot == 0) {
+                    done[0] = 1u;
+                } else {
+                    done[2] += 1u;
+                    if (trace && done[2] < trace_cap) trace[done[2]] = done[3];
+                }
+            }
+            *cnt = 0ull;
+            done[1] = 0u;
+        }
+    }
 }
 
-// One BFS level on one rank: compact the global frontier bitmap into a local queue (O(V/32)), grid
-// barrier, then expand it over the local (destination-owned) CSR with the hybrid mapping.  Discovered
-// owned vertices get their level and their bit in the next-frontier bitmap.
+// One BFS level on one rank.  The decision maker (Fig. 11 / the tuned rule) runs on the gathered
+// frontier's size (done[3], identical on every rank): for the queue working set the global frontier
+// bitmap is compacted into a local queue (O(V/32)), for the bitmap working set the tiles are the
+// bitmap's vertex ids directly (Fig. 9 line 1/2); either way the working set is expanded over the local
+// (destination-owned) CSR with the selected mapping, and discovered owned vertices get their level and
+// their bit in the next-frontier bitmap.  Device-side termination: a level launched after the frontier
+// became empty (done[0], raised by the previous finish kernel) returns at once, so the host enqueues
+// several levels without reading the frontier size.
 template <typename Off>
 __global__ void __launch_bounds__(BS, AG_MINB_BFS) dist_level_kernel(const TravArgs<Off> a, uint32_t L,
-                                                                     const uint32_t *front) {
+                                                                     const uint32_t *front, const unsigned *done) {
+    if (*(volatile const unsigned *)done) return;
     __shared__ TileSmem<Off, wq_cap<ALG_BFS>()> sm;
     Ctl *ctl = a.ctl;
     const uint32_t slot = 0;
     const uint32_t gtid = blockIdx.x * BS + threadIdx.x, gthreads = a.nblocks * BS;
-    compact_bitmap(front, a.nwords, a.q[0], &ctl->q_len[0], gtid >> 5, gthreads >> 5);
-    grid_barrier(ctl, a.nblocks);
-    const uint32_t qn = ld_relaxed(&ctl->q_len[0]);
+    const uint32_t n = *(volatile const unsigned *)(done + 3);
+    const uint8_t var = select_variant(a.pol, n, 0);
+    const uint32_t map = var >> 2, ws = var & 3u;
+    uint32_t qn = 0, tile_n = BS, ntiles;
+    if (ws == WS_QU) {
+        compact_bitmap(front, a.nwords, a.q[0], &ctl->q_len[0], gtid >> 5, gthreads >> 5);
+        grid_barrier(ctl, a.nblocks);
+        qn = ld_relaxed(&ctl->q_len[0]);
+        if (map != MAP_T) {
+            tile_n = (qn + 2 * a.nblocks - 1) / (2 * a.nblocks);
+            tile_n = tile_n < 1u ? 1u : (tile_n > (uint32_t)BS ? (uint32_t)BS : tile_n);
+        }
+        ntiles = (qn + tile_n - 1) / tile_n;
+    } else {
+        ntiles = (a.V + BS - 1) / BS;
+    }
     Ops<ALG_BFS, ORD_O, Off> ops(a, L, 0, true);
     ops.wbuf = sm.wq[threadIdx.x >> 5];
-    uint32_t tile_n = (qn + 2 * a.nblocks - 1) / (2 * a.nblocks);
-    tile_n = tile_n < 1u ? 1u : (tile_n > (uint32_t)BS ? (uint32_t)BS : tile_n);
-    const uint32_t ntiles = (qn + tile_n - 1) / tile_n;
+    const bool hubs = (map == MAP_H) && a.has_hubs;
+    const uint32_t s_idx = (map == MAP_W || (map == MAP_B && a.pol.cta_group == 32))
+                               ? (lane_id() * WARPS_PER_CTA + (threadIdx.x >> 5)) : threadIdx.x;
     uint32_t t = blockIdx.x;
     int par = 0;
     while (t < ntiles) {
-        if (threadIdx.x == 0) sm.tnext[par] = a.nblocks + atomicAdd(&ctl->tile_ctr[slot], 1u);
-        const uint32_t i = t * tile_n + threadIdx.x;
-        const bool valid = threadIdx.x < tile_n && i < qn;
-        const uint32_t u = valid ? a.q[0][i] : 0u;
-        if (__syncthreads_or(valid)) process_tile<true>(ops, sm, MAP_H, valid, u, 32u, a.has_hubs != 0, slot);
+        if (threadIdx.x == 0) sm.tnext[par] = ntiles > a.nblocks ? a.nblocks + atomicAdd(&ctl->tile_ctr[slot], 1u) : ntiles;
+        bool valid;
+        uint32_t u;
+        if (ws == WS_BM) {
+            u = t * BS + threadIdx.x;
+            valid = u < a.V && ((front[u >> 5] >> (u & 31)) & 1u);
+        } else {
+            const uint32_t i = t * tile_n + s_idx;
+            valid = s_idx < tile_n && i < qn;
+            u = valid ? a.q[0][i] : 0u;
+        }
+        if (__syncthreads_or(valid)) process_tile<false>(ops, sm, map, valid, u, a.pol.cta_group, hubs, slot);
         t = sm.tnext[par];
         par ^= 1;
     }
-    if (a.has_hubs) drain_hubs(ops, sm, slot);
+    if (hubs) drain_hubs(ops, sm, slot);
     ops.warp_flush(true);
     block_reduce_flush(ops, sm, ctl, slot);
 }
@@ -366,6 +427,8 @@ ag_status part_alloc(ag_graph_s *g, ag_comm_s *c) {
     if ((s = dev_alloc((void **)&d->d_next, (size_t)d->gwords * 4 + 128, g->device)) != AG_OK) return s;
     if ((s = dev_alloc((void **)&d->d_cnt, 64, g->device)) != AG_OK) return s;
     if (cudaMallocHost(&d->h_cnt, 64) != cudaSuccess) return set_error(AG_ERR_OOM, "pinned alloc");
+    if ((s = dev_alloc((void **)&d->d_done, 64, g->device)) != AG_OK) return s;
+    if (cudaMallocHost(&d->h_done, 64) != cudaSuccess) return set_error(AG_ERR_OOM, "pinned alloc");
     return AG_OK;
 }
 
@@ -395,10 +458,11 @@ struct LevelCfg {
 };
 
 template <typename Off>
-ag_status launch_level(ag_graph_s *g, uint32_t L, uint32_t *parent_local, cudaStream_t st) {
+ag_status launch_level(ag_graph_s *g, uint32_t L, uint32_t *parent_local, const ag_policy &pol, cudaStream_t st) {
     ag_dist_part *d = g->dist;
     TravArgs<Off> a;
     memset(&a, 0, sizeof a);
+    a.pol = resolve_policy(pol, *g);
     a.rp = (const Off *)g->d_rp;
     a.col = g->d_col;
     a.V = g->V;
@@ -420,7 +484,8 @@ ag_status launch_level(ag_graph_s *g, uint32_t L, uint32_t *parent_local, cudaSt
     a.nblocks = (uint32_t)(occ * g->num_sms);
     // reset the per-level counters of slot 0/1 (q_len, tile/hub scheduler)
     cudaMemsetAsync((char *)g->d_ctl + offsetof(Ctl, q_len), 0, offsetof(Ctl, it_edges) - offsetof(Ctl, q_len), st);
-    void *args[] = {(void *)&a, (void *)&L, (void *)&d->d_front};
+    const unsigned *done = d->d_done;
+    void *args[] = {(void *)&a, (void *)&L, (void *)&d->d_front, (void *)&done};
     cudaError_t e = cudaLaunchCooperativeKernel((const void *)fn, dim3(a.nblocks), dim3(BS), args, 0, st);
     note_launch(1);
     return cuda_status(e, "dist level");
@@ -495,9 +560,9 @@ ag_status run_sssp_round(ag_graph_s *g, const uint2 *list, uint32_t n, uint32_t 
                      : launch_sssp_round<unsigned long long>(g, list, n, ncin, cpar, hi, st);
 }
 
-ag_status run_level(ag_graph_s *g, uint32_t L, uint32_t *parent_local, cudaStream_t st) {
-    return g->offs32 ? launch_level<uint32_t>(g, L, parent_local, st)
-                     : launch_level<unsigned long long>(g, L, parent_local, st);
+ag_status run_level(ag_graph_s *g, uint32_t L, uint32_t *parent_local, const ag_policy &pol, cudaStream_t st) {
+    return g->offs32 ? launch_level<uint32_t>(g, L, parent_local, pol, st)
+                     : launch_level<unsigned long long>(g, L, parent_local, pol, st);
 }
 
 }  // namespace
@@ -685,15 +750,35 @@ ag_status ag_dist_graph_load_local(ag_comm c, uint32_t V, uint64_t E_local, cons
 namespace {
 
 // Lock-step driver over the participating ranks of THIS process (1 rank for NCCL, all for a group).
+// Device-side termination: per level the host ENQUEUES [level kernel, exchange, finish kernel] without
+// looking at the frontier; the finish kernel counts the gathered frontier on the device and raises
+// d_done when it is empty, after which the level kernels of later enqueued levels return at once.  The
+// host reads d_done once per BATCH of levels (4, doubling up to 64), not once per level.
 ag_status dist_bfs_driver(std::vector<ag_graph_s *> &parts, uint32_t src, uint32_t **levels_owned,
-                          uint32_t **parents_owned, ag_run_stats *stats, cudaStream_t st) {
+                          uint32_t **parents_owned, const ag_policy *pin, ag_run_stats *stats, cudaStream_t st) {
     const int P = (int)parts.size();
     ag_status s;
+    ag_policy pol;
+    if (pin) {
+        pol = *pin;
+    } else if ((s = ag_policy_default(&pol, parts[0]->device)) != AG_OK) {
+        return s;
+    }
+    if ((s = check_policy(&pol)) != AG_OK) return s;
+    const uint32_t tcap = stats && stats->trace_ws ? stats->trace_cap : 0;
     for (auto *g : parts) {
         cudaSetDevice(g->device);
         if ((s = dist_scratch(g)) != AG_OK) return s;
         if (parents_owned && !g->d_lpar && (s = dev_alloc((void **)&g->d_lpar, (size_t)g->V * 4 + 128, g->device)) != AG_OK)
             return s;
+        ag_dist_part *d = g->dist;
+        if (tcap > d->trace_cap) {
+            dev_free(d->d_trace, (size_t)d->trace_cap * 4 + 64, g->device);
+            d->d_trace = nullptr;
+            d->trace_cap = 0;
+            if ((s = dev_alloc((void **)&d->d_trace, (size_t)tcap * 4 + 64, g->device)) != AG_OK) return s;
+            d->trace_cap = tcap;
+        }
     }
     cudaEvent_t e0 = nullptr, e1 = nullptr;
     if (stats) {
@@ -702,52 +787,59 @@ ag_status dist_bfs_driver(std::vector<ag_graph_s *> &parts, uint32_t src, uint32
         cudaEventRecord(e0, st);
     }
     const uint32_t V = parts[0]->V;
+    static const uint32_t one = 1u;
     for (auto *g : parts) {
         ag_dist_part *d = g->dist;
         dist_init_kernel<<<g->num_sms * 4, 256, 0, st>>>(g->d_level, parents_owned ? g->d_lpar : nullptr, g->d_vis,
                                                         d->d_front, d->d_next, V, d->gwords, src);
         cudaMemsetAsync(g->d_ctl, 0, offsetof(Ctl, q_len), st);   // no-op for the barrier word (self-resetting)
         cudaMemsetAsync((char *)g->d_ctl + offsetof(Ctl, vexp), 0, 16, st);
+        cudaMemsetAsync(d->d_done, 0, 12, st);
+        cudaMemcpyAsync(d->d_done + 3, &one, 4, cudaMemcpyHostToDevice, st);   // |WS_0| = |{src}|
+        cudaMemsetAsync(d->d_cnt, 0, 8, st);
+        if (tcap) cudaMemcpyAsync(d->d_trace, &one, 4, cudaMemcpyHostToDevice, st);
         note_launch(1);
     }
-    uint32_t L = 0;
-    uint64_t front_n = 1;
-    uint32_t tcap = stats ? stats->trace_cap : 0;
-    for (;; ++L) {
-        if (stats && L < tcap && stats->trace_ws) stats->trace_ws[L] = (uint32_t)front_n;
-        for (auto *g : parts)
-            if ((s = run_level(g, L, parents_owned ? g->d_lpar : nullptr, st)) != AG_OK) return s;
-        // exchange: every rank contributes its owned slice of the next bitmap
-        if (P == 1 && parts[0]->dist->comm->nccl) {
-            ag_graph_s *g = parts[0];
-            ag_dist_part *d = g->dist;
-            ncclResult_t r = g_nccl.AllGather(d->d_next + (size_t)d->comm->rank * (d->S / 32), d->d_front, d->S / 8,
-                                              ncclUint8, d->comm->nccl, st);
-            if ((s = nccl_status(r, "ncclAllGather")) != AG_OK) return s;
-        } else {
-            for (auto *gd : parts) {
-                for (auto *gs : parts) {
-                    ag_dist_part *dd = gd->dist, *ds = gs->dist;
-                    const size_t off = (size_t)ds->comm->rank * (ds->S / 32);
-                    cudaMemcpyAsync(dd->d_front + off, ds->d_next + off, ds->S / 8, cudaMemcpyDeviceToDevice, st);
+    uint32_t L = 0, batch = 4;
+    bool fin = false;
+    while (!fin) {
+        for (uint32_t k = 0; k < batch; ++k, ++L) {
+            for (auto *g : parts)
+                if ((s = run_level(g, L, parents_owned ? g->d_lpar : nullptr, pol, st)) != AG_OK) return s;
+            // exchange: every rank contributes its owned slice of the next bitmap
+            if (P == 1 && parts[0]->dist->comm->nccl) {
+                ag_graph_s *g = parts[0];
+                ag_dist_part *d = g->dist;
+                ncclResult_t r = g_nccl.AllGather(d->d_next + (size_t)d->comm->rank * (d->S / 32), d->d_front, d->S / 8,
+                                                  ncclUint8, d->comm->nccl, st);
+                if ((s = nccl_status(r, "ncclAllGather")) != AG_OK) return s;
+            } else {
+                for (auto *gd : parts) {
+                    for (auto *gs : parts) {
+                        ag_dist_part *dd = gd->dist, *ds = gs->dist;
+                        const size_t off = (size_t)ds->comm->rank * (ds->S / 32);
+                        cudaMemcpyAsync(dd->d_front + off, ds->d_next + off, ds->S / 8, cudaMemcpyDeviceToDevice, st);
+                    }
                 }
             }
+            // every rank: clear its owned next slice, count the gathered frontier, decide termination
+            for (auto *g : parts) {
+                ag_dist_part *d = g->dist;
+                dist_level_finish_kernel<<<g->num_sms, 256, 0, st>>>(d->d_front, d->gwords,
+                                                                   d->d_next + (size_t)d->comm->rank * (d->S / 32), d->S / 32,
+                                                                   d->d_cnt, d->d_done, tcap ? d->d_trace : nullptr, tcap);
+                note_launch(1);
+            }
         }
-        // clear the owned next slices, count the gathered frontier (every rank sees the same count)
-        ag_graph_s *g0 = parts[0];
-        for (auto *g : parts) {
-            ag_dist_part *d = g->dist;
-            cudaMemsetAsync(d->d_next + (size_t)d->comm->rank * (d->S / 32), 0, d->S / 8, st);
-        }
-        cudaMemsetAsync(g0->dist->d_cnt, 0, 8, st);
-        popcount_kernel<<<g0->num_sms * 2, 256, 0, st>>>(g0->dist->d_front, g0->dist->gwords, g0->dist->d_cnt);
-        note_launch(1);
-        cudaMemcpyAsync(g0->dist->h_cnt, g0->dist->d_cnt, 8, cudaMemcpyDeviceToHost, st);
+        ag_dist_part *d0 = parts[0]->dist;
+        cudaMemcpyAsync(d0->h_done, d0->d_done, 16, cudaMemcpyDeviceToHost, st);
         cudaError_t ce = cudaStreamSynchronize(st);
         if (ce != cudaSuccess) return cuda_status(ce, "dist level");
-        front_n = *g0->dist->h_cnt;
-        if (front_n == 0 || L > V) break;
+        fin = d0->h_done[0] != 0;
+        if (!fin && L > V + 1) return set_error(AG_ERR_CUDA, "dist bfs did not terminate");
+        batch = batch < 64 ? 2 * batch : 64;
     }
+    const uint32_t levels = parts[0]->dist->h_done[2] + 1;   // nonempty frontiers, {src} included
     // outputs: owned slices of level / parent
     for (int r = 0; r < P; ++r) {
         ag_graph_s *g = parts[r];
@@ -766,7 +858,7 @@ ag_status dist_bfs_driver(std::vector<ag_graph_s *> &parts, uint32_t src, uint32
         cudaEventElapsedTime(&ms, e0, e1);
         cudaEventDestroy(e0);
         cudaEventDestroy(e1);
-        stats->iterations = L + 1;
+        stats->iterations = levels;
         stats->device_ms = ms;
         unsigned long long vx = 0, ex = 0;
         for (auto *g : parts) {
@@ -777,7 +869,9 @@ ag_status dist_bfs_driver(std::vector<ag_graph_s *> &parts, uint32_t src, uint32
         }
         stats->vertices_expanded = vx;  // summed over the ranks of this process
         stats->edges_inspected = ex;
-        stats->trace_len = (L + 1) < tcap ? (L + 1) : tcap;
+        const uint32_t n = levels < tcap ? levels : tcap;
+        stats->trace_len = n;
+        if (n) cudaMemcpy(stats->trace_ws, parts[0]->dist->d_trace, (size_t)n * 4, cudaMemcpyDeviceToHost);
     }
     return AG_OK;
 }
@@ -928,7 +1022,6 @@ extern "C" {
 
 ag_status ag_dist_bfs(ag_graph local, uint32_t src, uint32_t *levels_owned, uint32_t *parents_owned,
                       const ag_policy *policy, ag_run_stats *stats, void *stream) {
-    (void)policy;
     if (!local || !local->dist) return set_error(AG_ERR_INVALID_ARG, "not a distributed graph");
     if (src >= local->V) return set_error(AG_ERR_SRC_RANGE, "src %u >= V %u", src, local->V);
     if (stats && stats->struct_size != sizeof(ag_run_stats)) return set_error(AG_ERR_INVALID_ARG, "stats size");
@@ -937,7 +1030,7 @@ ag_status ag_dist_bfs(ag_graph local, uint32_t src, uint32_t *levels_owned, uint
     uint32_t *lv[1] = {levels_owned};
     uint32_t *pa[1] = {parents_owned};
     cudaSetDevice(local->device);
-    return dist_bfs_driver(parts, src, lv, parents_owned ? pa : nullptr, stats, (cudaStream_t)stream);
+    return dist_bfs_driver(parts, src, lv, parents_owned ? pa : nullptr, policy, stats, (cudaStream_t)stream);
 }
 
 ag_status ag_dist_bfs_group(ag_graph *locals, int world, uint32_t src, uint32_t **levels_owned,
@@ -952,7 +1045,7 @@ ag_status ag_dist_bfs_group(ag_graph *locals, int world, uint32_t src, uint32_t 
     if (src >= parts[0]->V) return set_error(AG_ERR_SRC_RANGE, "src out of range");
     if (stats && stats->struct_size != sizeof(ag_run_stats)) return set_error(AG_ERR_INVALID_ARG, "stats size");
     cudaSetDevice(parts[0]->device);
-    return dist_bfs_driver(parts, src, levels_owned, parents_owned, stats, (cudaStream_t)stream);
+    return dist_bfs_driver(parts, src, levels_owned, parents_owned, nullptr, stats, (cudaStream_t)stream);
 }
 
 ag_status ag_dist_sssp(ag_graph local, uint32_t src, uint32_t *dist_owned, uint32_t *parents_owned,

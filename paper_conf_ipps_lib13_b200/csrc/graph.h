@@ -71,6 +71,9 @@ bool is_device_ptr(const void *p);
 ag_status check_device(int device, int *num_sms);
 void note_launch(unsigned n);
 void dist_graph_release(ag_graph_s *g);
+struct DevPolicy;
+DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g);
+ag_status check_policy(const ag_policy *p);
 void build_degree_order(const uint64_t *rp64, uint32_t V, unsigned long long *keys, unsigned long long *keys2, void *tmp,
                         size_t tmp_bytes, uint32_t *perm, uint32_t *inv, uint64_t *ndeg, uint64_t *nrp, int sms,
                         cudaStream_t st);

@@ -83,6 +83,10 @@ struct TravArgs {
 #ifndef AG_BLIND
 #define AG_BLIND 1
 #endif
+#ifndef AG_DEDUP
+#define AG_DEDUP 0
+#endif
+constexpr bool freeo_static = false;
 // per-warp staging capacity: one batch appends at most 32 x (edges per thread per batch), plus < 32 left over
 // (sized per algorithm: the smaller SSSP buffer lets the L1/shared carveout leave more L1 to the status
 // gathers, see launch_traverse)
@@ -105,6 +109,7 @@ struct __align__(16) TileSmem {
     unsigned long long red64[2][WARPS_PER_CTA];
     uint32_t red32[2][WARPS_PER_CTA];
     int redi[WARPS_PER_CTA];
+    uint32_t redrx[WARPS_PER_CTA];
     uint32_t redany[WARPS_PER_CTA];
     uint32_t tnext[2];
     uint32_t bcast;
@@ -132,6 +137,7 @@ struct Ops {
     uint32_t *wbuf;         // this warp's staging buffer in shared memory (hybrid mapping)
     uint32_t wfill;         // its fill level (warp-uniform)
     unsigned long long ne, nv;
+    uint32_t reexp = 0;     // SSSP with an adaptive order: re-expansions (measured redundancy)
     uint32_t vmin;
     int dpend;
     bool ovf;
@@ -142,7 +148,7 @@ struct Ops {
     uint32_t hdeg = HUB_DEG, hchunk = HUB_CHUNK;   // hub-task degree threshold and chunk (per iteration)
 
     __device__ Ops(const TravArgs<Off> &a_, uint32_t it_, uint64_t hi_, bool append_)
-        : a(a_), it(it_), hi(hi_), append_next(append_), fenced(ALG == ALG_SSSP && ORD == ORD_O && a_.pol.delta > 1),
+        : a(a_), it(it_), hi(hi_), append_next(append_), fenced(ALG == ALG_SSSP && ORD == ORD_O && (a_.pol.delta > 1 || a_.pol.adapt)),
           pol_stream(policy_evict_first()), pol_keep(policy_evict_last()), wbuf(nullptr), wfill(0), ne(0), nv(0),
           vmin(INF), dpend(0), ovf(false), nact(a_.nblocks) {
         const uint32_t sn = (it_ + 1) % 3;
@@ -215,6 +221,10 @@ struct Ops {
             deg = (uint32_t)(re - rb);
             nv += 1;
             ne += deg;
+            if (ALG == ALG_SSSP && a.pol.adapt && !a.ulist) {   // first expansion of u in this query?
+                const uint32_t m = 1u << (u & 31);
+                if (atomicOr(&a.vis[u >> 5], m) & m) reexp += 1;
+            }
         } else {
             deg = 0;
         }
@@ -327,6 +337,37 @@ struct Ops {
             }
         }
         if (CONV && !__any_sync(0xffffffffu, cm != 0)) return 0u;
+#if AG_DEDUP
+        // warp-level dedup (all lanes converged): lanes of this warp that would issue an atomic on the SAME
+        // target v in slot j are grouped with __match_any_sync; only the lane with the smallest candidate
+        // value (SSSP: distance, ties -> lowest lane; BFS / CC: the lowest lane) keeps its atomic.  The
+        // dropped candidates could not have won against it, so the results are unchanged; the atomics on
+        // hot targets (hubs, whose lists every warp of a hub task shares) are no longer serialised per lane.
+        if constexpr (CONV && !freeo_static) {
+            if (!freeo) {
+                const unsigned lane = lane_id();
+#pragma unroll
+                for (int j = 0; j < NB; ++j) {
+                    const bool c = (cm >> j) & 1u;
+                    const unsigned act = __ballot_sync(0xffffffffu, c);
+                    if (__popc(act) < 2) continue;
+                    if (c) {
+                        const unsigned grp = __match_any_sync(act, v[j]);
+                        if (grp != (1u << lane)) {
+                            unsigned keep;
+                            if constexpr (ALG == ALG_SSSP || ALG == ALG_CC) {
+                                const uint32_t mn = __reduce_min_sync(grp, (uint32_t)nd[j]);
+                                keep = __ballot_sync(grp, (uint32_t)nd[j] == mn);
+                            } else {
+                                keep = grp;
+                            }
+                            if ((int)lane != __ffs(keep) - 1) cm &= ~(1u << j);
+                        }
+                    }
+                }
+            }
+        }
+#endif
         if (freeo) {
             // free output: every candidate marks v in the next bitmap with a reduction that returns
             // nothing (the update vector, 22.s13-14); BFS levels are assigned when the next iteration
@@ -509,27 +550,6 @@ struct Ops {
                 vv[j * QE + k] = pv[j];
             }
         }
-#if defined(AG_EXPERIMENT) && (AG_EXPERIMENT == 11 || AG_EXPERIMENT == 12)
-        // marginal-cost experiments (same frontiers, extra work): 11 repeats the 128-bit CSR loads,
-        // 12 repeats the CSR loads and the status gathers
-        {
-            uint32_t acc = 0;
-#pragma unroll
-            for (int j = 0; j < NQ; ++j) {
-                uint4 c = pok[j] ? ld_stream4(reinterpret_cast<const uint4 *>(
-                                                  (ALG == ALG_SSSP) ? (const void *)(a.cw + pq[j] * QE + 0)
-                                                                    : (const void *)(a.col + pq[j] * QE + 0)),
-                                              pol_keep)
-                                 : make_uint4(0u, 0u, 0u, 0u);
-                if (AG_EXPERIMENT == 12) {
-                    if (pok[j]) acc += status(c.x) + status(c.z) + ((ALG == ALG_SSSP) ? 0u : status(c.y) + status(c.w));
-                } else {
-                    acc += c.x ^ c.y ^ c.z ^ c.w;
-                }
-            }
-            if (acc == 0x9E3779B1u) ovf = true;
-        }
-#endif
         batch_vals<N, true>(uu, vv, v, wt, ok);
     }
 
@@ -626,6 +646,7 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, SmT 
     unsigned long long ne = warp_sum(ops.ne), nv = warp_sum(ops.nv);
     uint32_t vmin = warp_min(ops.vmin);
     int dp = warp_sum(ops.dpend);
+    const uint32_t rx = warp_sum(ops.reexp);
     unsigned ovf = __any_sync(0xffffffffu, ops.ovf);
     unsigned anyw = __any_sync(0xffffffffu, ops.any);
     if (lane == 0) {
@@ -635,13 +656,16 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, SmT 
         sm.red32[0][wid] = vmin;
         sm.red32[1][wid] = ovf;
         sm.redi[wid] = dp;
+        sm.redrx[wid] = rx;
     }
     __syncthreads();
     if (threadIdx.x == 0) {
         unsigned long long se = 0, sv = 0;
         uint32_t mn = INF, ov = 0, an = 0;
         int sd = 0;
+        uint32_t srx = 0;
         for (int i = 0; i < WARPS_PER_CTA; ++i) {
+            srx += sm.redrx[i];
             an |= sm.redany[i];
             se += sm.red64[0][i];
             sv += sm.red64[1][i];
@@ -651,9 +675,13 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, SmT 
         }
         if (se) {
             atomicAdd(&ctl->eexp, se);
-            if (ops.a.trace_edges) atomicAdd(&ctl->it_edges[slot], se);
+            atomicAdd(&ctl->it_edges[slot], se);   // m_F of this working set (selector input, trace)
         }
-        if (sv) atomicAdd(&ctl->vexp, sv);
+        if (sv) {
+            atomicAdd(&ctl->vexp, sv);
+            atomicAdd(&ctl->it_nv[slot], sv);
+        }
+        if (srx) atomicAdd(&ctl->it_reexp[slot], srx);
         if (ALG == ALG_SSSP) {
             if (mn != INF) atomicMin(&ctl->next_min[(slot + 1) % 3], mn);
             if (ORD == ORD_O && sd) atomicAdd(&ctl->pend_count, (unsigned)sd);
@@ -776,18 +804,6 @@ __device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, SmT &sm, u
             plo[j] = bo;
             phi[j] = bo + sm.deg[lo];
             pq[j] = bo / QE + (p - sm.scan[lo]);   // aligned piece index
-#if defined(AG_EXPERIMENT) && AG_EXPERIMENT == 13   // marginal cost of the owner search: search twice
-            {
-                uint32_t lo2 = 0, hi2 = BS;
-                const uint32_t p2 = p ^ (uint32_t)(pq[j] & 1);
-#pragma unroll
-                for (int step = 0; step < LOG_BS; ++step) {
-                    const uint32_t mid = (lo2 + hi2) >> 1;
-                    if (sm.scan[mid] <= p2) lo2 = mid; else hi2 = mid;
-                }
-                if (lo2 == 0xFFFFu) ops.ovf = true;
-            }
-#endif
         }
         ops.template pieces<QB>(pu, pv, pq, plo, phi, pok);
     }
@@ -1024,6 +1040,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             a.bm[2][wi] = 0u;
         }
         if (ALG == ALG_BFS) a.vis[wi] = (wi == sword) ? sbit : 0u;
+        if (ALG == ALG_SSSP && a.pol.adapt) a.vis[wi] = 0u;   // "expanded before" bits (redundancy measure)
     }
     if (gtid == 0) {
         if (ALG != ALG_CC) a.q[0][0] = src;
@@ -1035,6 +1052,8 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             ctl->hub_head[s] = 0;
             ctl->stage_done[s] = 0;
             ctl->it_edges[s] = 0;
+            ctl->it_nv[s] = 0;
+            ctl->it_reexp[s] = 0;
             ctl->free_any[s] = 0;
         }
         ctl->pend_count = 1;
@@ -1076,6 +1095,10 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     uint32_t prev_ws = WS_QU;   // representation used in the previous iteration
     uint8_t prev_var = 0;
     uint32_t n_prev = 0;
+    // SSSP order axis (NEXT-3): the unordered deferral window / the ordered bucket width; adapted per
+    // iteration from the measured redundancy when the policy asks for it (identical on every CTA: the
+    // inputs are global counters, and a parked CTA receives the current value when woken)
+    uint32_t win = ROT ? a.pol.window : a.pol.delta;
     uint32_t it = 0;
     bool in_raw = false;   // this iteration's working set is the raw bitmap of a free-output iteration
     for (;; ++it) {
@@ -1097,6 +1120,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
                     ctl->wake_it = it;
                     ctl->wake_n = n;
                     ctl->wake_nprev = n_prev;
+                    ctl->wake_win = win;
                     __threadfence();
                     st_release(&ctl->wake_gen, wgen + 1u);
                 }
@@ -1111,12 +1135,14 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
                         sm.red32[1][0] = ld_relaxed(&ctl->wake_it);
                         sm.red32[1][1] = ld_relaxed(&ctl->wake_n);
                         sm.red32[1][2] = ld_relaxed(&ctl->wake_nprev);
+                        sm.red32[1][3] = ld_relaxed(&ctl->wake_win);
                     }
                     __syncthreads();
                     wgen += 1u;
                     it = sm.red32[1][0];
                     n = sm.red32[1][1];
                     n_prev = sm.red32[1][2];
+                    win = sm.red32[1][3];
                     __syncthreads();
                     nact = a.nblocks;
                     prev_var = 0;
@@ -1128,9 +1154,16 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         const uint32_t gact = nact * BS;   // threads taking part (grid-strided loops of this iteration)
         AG_PROF_MARK(it, 0);
         // decision maker, re-evaluated every sample_every iterations (inspector sampling, 26.s7-9)
-        const uint8_t var = (it % a.pol.sample_every == 0 || prev_var == 0) ? select_variant(a.pol, n, 0) : prev_var;
+        // m_F estimate for the selector: |WS| x the previous frontier's average out-degree (the graph's
+        // average at it = 0) — the inspector's working-set statistic (26.s4-7)
+        // (every CTA reads the same global counter: the decision must be grid-uniform)
+        const uint64_t mf_prev = it ? ld_relaxed64(&ctl->it_edges[(it + 2) % 3]) : 0ull;
+        const uint64_t mf = n_prev ? (uint64_t)n * mf_prev / n_prev : (uint64_t)n * ((a.pol.E + a.V - 1) / a.V);
+        const uint8_t var = (it % a.pol.sample_every == 0 || prev_var == 0) ? select_variant(a.pol, n, mf) : prev_var;
         const uint32_t map = TUNED ? ((var >> 2) == MAP_T ? (uint32_t)MAP_T : (uint32_t)MAP_H) : (var >> 2);
-        const uint32_t ws = TUNED ? (uint32_t)WS_QU : (var & 3u);
+        // tuned kernels: the queue, except the ordered-SSSP pending set, whose bitmap tier the selector
+        // picks once the set is dense (select_variant)
+        const uint32_t ws = (TUNED && ROT) ? (uint32_t)WS_QU : (var & 3u);
         if (vid == 0 && threadIdx.x == 0) {
             if (it < a.trace_cap && a.trace_ws) {
                 a.trace_ws[it] = n;
@@ -1145,20 +1178,31 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             ctl->hub_tail[rs] = 0;
             ctl->hub_head[rs] = 0;
             ctl->stage_done[rs] = 0;
-            ctl->it_edges[rs] = 0;
+            ctl->it_edges[(it + 1) % 3] = 0;   // (slot it%3 is still read after this iteration's barrier)
+            ctl->it_nv[(it + 1) % 3] = 0;
+            ctl->it_reexp[(it + 1) % 3] = 0;
             ctl->free_any[rs] = 0;
         }
 
         uint64_t hi = ~0ull;
         bool append = true;
         uint32_t qn = n;
-        if (ALG == ALG_SSSP && ROT && a.pol.window) {
+        if (ALG == ALG_SSSP && a.pol.adapt && it > 0) {
+            // redundancy of the previous iteration: re-expanded / expanded.  Much waste -> a narrower
+            // window (more ordered, fewer redundant relaxations); little waste -> a wider one (more
+            // parallel work per iteration, fewer iterations).  Results are unchanged either way.
+            const unsigned long long nvp = ld_relaxed64(&ctl->it_nv[(it + 2) % 3]);
+            const uint32_t rxp = ld_relaxed(&ctl->it_reexp[(it + 2) % 3]);
+            if ((unsigned long long)rxp * 4ull > nvp) win = win > 1u ? win >> 1 : 1u;
+            else if ((unsigned long long)rxp * 16ull < nvp && win < a.pol.win_max) win <<= 1;
+        }
+        if (ALG == ALG_SSSP && ROT && win) {
             const uint32_t lo = ld_relaxed(&ctl->next_min[slot]);
-            hi = (uint64_t)lo + a.pol.window;
+            hi = (uint64_t)lo + win;
         }
         if (!ROT) {
             const uint32_t lo = ld_relaxed(&ctl->next_min[slot]);
-            hi = (uint64_t)lo + a.pol.delta;
+            hi = (uint64_t)lo + win;
             append = (ws == WS_QU);
             if (ws == WS_QU) {
                 if (prev_ws != WS_QU) {
@@ -1291,15 +1335,6 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     // exact overflow test (rare path: only when a relaxation exceeded MAX_FINITE): a reachable vertex
     // left at INF behind a finite one.  The packed state is final here (every CTA passed the barrier
     // that ended the last iteration, or was parked without writing), so no further barrier is needed.
-    if (ALG == ALG_SSSP && !a.ulist && ld_relaxed(&ctl->overflow)) {
-        bool bad = false;
-        for (uint32_t u = gtid; u < a.V && !bad; u += gthreads) {
-            if ((a.P[u] >> 32) == INF) continue;
-            for (Off e = a.rp[u]; e < a.rp[u + 1]; ++e)
-                if ((a.P[a.cw[e].x] >> 32) == INF) { bad = true; break; }
-        }
-        if (bad) atomicOr(&ctl->sticky, 1u);
-    }
     if (ALG == ALG_SSSP) {  // unpack (dist, parent) into the caller's arrays (caller ids)
         for (uint32_t v = gtid; v < a.V; v += gthreads) {
             unsigned long long pv = a.P[a.inv ? a.inv[v] : v];

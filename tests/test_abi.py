@@ -107,3 +107,34 @@ def test_ag_select_forced_axes(L):
     assert A.select(p, info, 1, 0) == A.variant(A.MAP_WARP, A.WS_BITMAP)
     p.mapping, p.workset = A.MAP_AUTO, A.WS_QUEUE
     assert A.select(p, info, 10**6, 0) == A.variant(A.MAP_THREAD, A.WS_QUEUE)
+
+
+def _tuned_policy(order=0):
+    p = _paper_policy()
+    p.kind = A.POLICY_TUNED
+    p.order = order
+    return p
+
+
+def test_ag_select_tuned_rule(L):
+    """The tuned decision maker (common.cuh select_variant) as a pure function of (|WS|,
+    m_F, graph): thread mapping only for small, low-degree working sets of a graph without long lists;
+    the bitmap only for a dense ordered-SSSP pending set (>= V/32); the hybrid queue otherwise."""
+    info = A.GraphInfo()
+    info.num_vertices, info.num_edges, info.max_deg = 1 << 20, 8 << 20, 40     # ER-like: max degree 40
+    p = _tuned_policy()
+    T, H, QU, BM = A.MAP_THREAD, A.MAP_HYBRID, A.WS_QUEUE, A.WS_BITMAP
+    assert A.select(p, info, 1000, 8000) == A.variant(T, QU)           # small, avg degree 8
+    assert A.select(p, info, 1000, 16000) == A.variant(T, QU)          # m_F = 16 |WS|: still low
+    assert A.select(p, info, 1000, 16001) == A.variant(H, QU)          # above: load-balanced
+    assert A.select(p, info, 65535, 8 * 65535) == A.variant(T, QU)
+    assert A.select(p, info, 65536, 8 * 65536) == A.variant(H, QU)     # big working set
+    info.max_deg = 65                                                   # one long list: straggler risk
+    assert A.select(p, info, 1000, 8000) == A.variant(H, QU)
+    # unordered: never the bitmap, however dense
+    assert A.select(p, info, 1 << 20, 8 << 20) == A.variant(H, QU)
+    # ordered SSSP pending set: bitmap from V/32 on
+    po = _tuned_policy(order=A.ORDERED)
+    V32 = (1 << 20) // 32
+    assert A.select(po, info, V32 - 1, 8 * V32) == A.variant(H, QU)
+    assert A.select(po, info, V32, 8 * V32) == A.variant(H, BM)

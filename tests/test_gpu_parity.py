@@ -326,13 +326,12 @@ def test_torch_allocator_hook():
 
 
 # ------------------------------------------------------------------------------------------------
-# small-frontier mode (tuned kernels on graphs without hub tasks): iterations with |WS| < t_small run
+# small-frontier mode (tuned kernels on graphs without hub tasks): iterations with |WS| < small_ws run
 # on one CTA per SM while the rest park; thresholds forced low so the group shrinks and grows many
-# times inside one traversal (env AG_SMALL_WS is read per query)
+# times inside one traversal (policy field small_ws)
 # ------------------------------------------------------------------------------------------------
-@pytest.mark.parametrize("t_small", ["1", "8", "100", "5000", "0"])
-def test_small_frontier_mode_transitions(t_small, monkeypatch):
-    monkeypatch.setenv("AG_SMALL_WS", t_small)
+@pytest.mark.parametrize("small_ws", [1, 8, 100, 5000, 0xFFFFFFFF])
+def test_small_frontier_mode_transitions(small_ws):
     graphs = [aggen.config("C1"), aggen.with_weights(aggen.grid(60, 50), seed=9, wmax=100),
               aggen.with_weights(aggen.er(5000, 20000, seed=4), seed=5, wmax=100),
               aggen.random_graph(3000, 9000, seed=12)]
@@ -341,20 +340,36 @@ def test_small_frontier_mode_transitions(t_small, monkeypatch):
             G = A.Graph.from_csr(g, layout=layout)
             lab = oracle.cc(g)
             for s in sorted(set(int(x) for x in aggen.sources(g, 2)) | {0}):
-                check_bfs(g, G, s, pol(0), want_parents=False)
-                check_bfs(g, G, s, pol(0))
-                check_bfs(g, G, s, pol(1))
-                check_sssp(g, G, s, pol(0))
-                check_sssp(g, G, s, pol(0, free_ppm=1000000))
-                check_sssp(g, G, s, pol(1, delta=4))
-            assert np.array_equal(G.cc(policy=pol(0))[0], lab)
-            assert np.array_equal(G.cc(policy=pol(0, free_ppm=1000000))[0], lab)
+                check_bfs(g, G, s, pol(0, small_ws=small_ws), want_parents=False)
+                check_bfs(g, G, s, pol(0, small_ws=small_ws))
+                check_bfs(g, G, s, pol(1, small_ws=small_ws))
+                check_sssp(g, G, s, pol(0, small_ws=small_ws))
+                check_sssp(g, G, s, pol(0, small_ws=small_ws, free_ppm=1000000))
+                check_sssp(g, G, s, pol(1, delta=4, small_ws=small_ws))
+            assert np.array_equal(G.cc(policy=pol(0, small_ws=small_ws))[0], lab)
+            assert np.array_equal(G.cc(policy=pol(0, small_ws=small_ws, free_ppm=1000000))[0], lab)
+
+
+def test_ordered_sssp_bitmap_tier():
+    """The tuned policy switches the ordered-SSSP pending set between the bitmap (>= V/32 pending) and
+    the queue per iteration (select_variant); both representations and every switch must give the
+    Dijkstra distances."""
+    for g in (aggen.with_weights(aggen.er(20000, 100000, seed=4), seed=5, wmax=100),
+              aggen.config("C1"), aggen.with_weights(aggen.grid(80, 60), seed=9, wmax=100)):
+        G = A.Graph.from_csr(g)
+        for s in aggen.sources(g, 2):
+            for delta in (1, 16):
+                st = check_sssp(g, G, int(s), pol(1, delta=delta))
+                assert st.iterations >= 1
+            out, _, st = G.sssp(int(s), policy=pol(1), stats=True, trace_cap=1 << 16)
+            v = set(int(x) & 3 for x in st.trace_variant)
+            if g.V == 20000:
+                assert v == {1, 2}, v   # both tiers used on the ER graph
 
 
 @pytest.mark.parametrize("cfg", ["C3", "C4"])
-def test_small_frontier_mode_full_size(cfg, monkeypatch):
-    """Default threshold on the latency-bound grid and on ER (frontier grows through t_small and back)."""
-    monkeypatch.delenv("AG_SMALL_WS", raising=False)
+def test_default_policy_full_size_no_parents(cfg):
+    """bench.py's calls on the latency-bound grid and on ER (free output, no parents)."""
     g = aggen.config(cfg)
     G = A.Graph.from_csr(g)
     for s in [int(x) for x in aggen.sources(g, 1)]:
@@ -491,3 +506,36 @@ def test_deferred_overflow_is_sticky_across_queries():
     with pytest.raises(A.AgError) as e:           # the earlier overflow survives the later good query
         G.check()
     assert e.value.status == "AG_ERR_OVERFLOW"
+
+
+@pytest.mark.parametrize("mode", ["window", "delta"])
+def test_adaptive_order_axis(mode):
+    """NEXT-3: the SSSP order axis adapted per iteration from the measured re-expansion ratio — the
+    unordered deferral window (sssp_window = AG_WINDOW_ADAPTIVE) or the ordered bucket width
+    (delta = 0) — reorders the work but never changes the distances."""
+    graphs = [aggen.config("C1"), aggen.with_weights(aggen.grid(60, 50), seed=9, wmax=100),
+              aggen.with_weights(aggen.er(5000, 20000, seed=4), seed=5, wmax=100),
+              aggen.random_graph(2000, 12000, seed=21, wmax=1000),
+              aggen.with_weights(aggen.star(20000))]
+    for g in graphs:
+        for layout in (1, 2):
+            G = A.Graph.from_csr(g, layout=layout)
+            for s in sorted(set(int(x) for x in aggen.sources(g, 2)) | {0}):
+                if mode == "window":
+                    check_sssp(g, G, s, pol(0, sssp_window=A.WINDOW_ADAPTIVE))
+                    check_sssp(g, G, s, pol(0, sssp_window=A.WINDOW_ADAPTIVE, free_ppm=1000000))
+                    check_sssp(g, G, s, pol(0, 1, 2, sssp_window=A.WINDOW_ADAPTIVE))
+                else:
+                    check_sssp(g, G, s, pol(1, delta=0))
+                    check_sssp(g, G, s, pol(1, 4, 1, delta=0))
+                    check_sssp(g, G, s, pol(1, 1, 2, delta=0))
+
+
+@pytest.mark.parametrize("cfg", ["C3p", "C4"])
+def test_adaptive_order_axis_full_size(cfg):
+    g = aggen.config(cfg)
+    G = A.Graph.from_csr(g)
+    s = int(aggen.sources(g, 1, seed=5)[0])
+    d = oracle.dijkstra(g, s, want_parents=False)[0]
+    check_sssp(g, G, s, pol(0, sssp_window=A.WINDOW_ADAPTIVE), expect_dist=d)
+    check_sssp(g, G, s, pol(1, delta=0), expect_dist=d)
