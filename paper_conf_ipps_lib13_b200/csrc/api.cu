@@ -411,7 +411,13 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
     // Unordered BFS on degree-layout (hub) graphs runs the tuned policy's decisions (hybrid mapping,
     // queue) in the general specialisation: C2 median 0.575 -> 0.566 ms, mean 0.588 -> 0.565 ms over
     // 16 sources (profiles/r01_bfs_tuned_probe.txt; cause in the tuned specialisation not found).
-    const bool tuned = a.pol.kind == AG_POLICY_TUNED && a.pol.force_map == 0 && a.pol.force_ws == 0 &&
+    // A forced variant the tuned specialisation implements (thread or hybrid mapping over the queue; for the
+    // ordered-SSSP pending set also the bitmap) runs in it too, with the same engine features as the
+    // adaptive runs (free output, small-frontier mode), so static-vs-adaptive is like for like there.
+    const bool tuned_map = a.pol.force_map == 0 || a.pol.force_map == MAP_T || a.pol.force_map == MAP_H;
+    const bool tuned_ws = a.pol.force_ws == 0 || a.pol.force_ws == WS_QU ||
+                          (ALG == ALG_SSSP && ORD == ORD_O && a.pol.force_ws == WS_BM);
+    const bool tuned = a.pol.kind == AG_POLICY_TUNED && tuned_map && tuned_ws &&
                        !(ALG == ALG_BFS && ORD == ORD_U && g->info.layout == AG_LAYOUT_DEGREE);
     auto fn = tuned ? traverse_kernel<ALG, ORD, Off, true> : traverse_kernel<ALG, ORD, Off, false>;
     const size_t dyn = 0;

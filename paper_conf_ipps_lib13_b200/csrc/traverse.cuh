@@ -83,10 +83,6 @@ struct TravArgs {
 #ifndef AG_BLIND
 #define AG_BLIND 1
 #endif
-#ifndef AG_DEDUP
-#define AG_DEDUP 0
-#endif
-constexpr bool freeo_static = false;
 // per-warp staging capacity: one batch appends at most 32 x (edges per thread per batch), plus < 32 left over
 // (sized per algorithm: the smaller SSSP buffer lets the L1/shared carveout leave more L1 to the status
 // gathers, see launch_traverse)
@@ -337,37 +333,7 @@ struct Ops {
             }
         }
         if (CONV && !__any_sync(0xffffffffu, cm != 0)) return 0u;
-#if AG_DEDUP
-        // warp-level dedup (all lanes converged): lanes of this warp that would issue an atomic on the SAME
-        // target v in slot j are grouped with __match_any_sync; only the lane with the smallest candidate
-        // value (SSSP: distance, ties -> lowest lane; BFS / CC: the lowest lane) keeps its atomic.  The
-        // dropped candidates could not have won against it, so the results are unchanged; the atomics on
-        // hot targets (hubs, whose lists every warp of a hub task shares) are no longer serialised per lane.
-        if constexpr (CONV && !freeo_static) {
-            if (!freeo) {
-                const unsigned lane = lane_id();
-#pragma unroll
-                for (int j = 0; j < NB; ++j) {
-                    const bool c = (cm >> j) & 1u;
-                    const unsigned act = __ballot_sync(0xffffffffu, c);
-                    if (__popc(act) < 2) continue;
-                    if (c) {
-                        const unsigned grp = __match_any_sync(act, v[j]);
-                        if (grp != (1u << lane)) {
-                            unsigned keep;
-                            if constexpr (ALG == ALG_SSSP || ALG == ALG_CC) {
-                                const uint32_t mn = __reduce_min_sync(grp, (uint32_t)nd[j]);
-                                keep = __ballot_sync(grp, (uint32_t)nd[j] == mn);
-                            } else {
-                                keep = grp;
-                            }
-                            if ((int)lane != __ffs(keep) - 1) cm &= ~(1u << j);
-                        }
-                    }
-                }
-            }
-        }
-#endif
+
         if (freeo) {
             // free output: every candidate marks v in the next bitmap with a reduction that returns
             // nothing (the update vector, 22.s13-14); BFS levels are assigned when the next iteration
@@ -899,6 +865,7 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, SmT &sm, uin
     }
 }
 
+
 // Warp-cooperative, in-order emission of the set bits of the warp's 32 consecutive words (word w0 + lane,
 // popcount c, inclusive warp count x, warp total tot) as vertex ids out[0 .. tot): output i goes to lane
 // i % 32, which finds the owning word (binary search over the lanes' inclusive counts, by shuffles) and
@@ -1099,6 +1066,8 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     // iteration from the measured redundancy when the policy asks for it (identical on every CTA: the
     // inputs are global counters, and a parked CTA receives the current value when woken)
     uint32_t win = ROT ? a.pol.window : a.pol.delta;
+    // (unordered: never below the start value — narrower windows measured slower on C2/C3/C4)
+    const uint32_t win_min = ROT ? (win ? win : 1u) : 1u;
     uint32_t it = 0;
     bool in_raw = false;   // this iteration's working set is the raw bitmap of a free-output iteration
     for (;; ++it) {
@@ -1193,7 +1162,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             // parallel work per iteration, fewer iterations).  Results are unchanged either way.
             const unsigned long long nvp = ld_relaxed64(&ctl->it_nv[(it + 2) % 3]);
             const uint32_t rxp = ld_relaxed(&ctl->it_reexp[(it + 2) % 3]);
-            if ((unsigned long long)rxp * 4ull > nvp) win = win > 1u ? win >> 1 : 1u;
+            if ((unsigned long long)rxp * 4ull > nvp) win = win > win_min ? win >> 1 : win_min;
             else if ((unsigned long long)rxp * 16ull < nvp && win < a.pol.win_max) win <<= 1;
         }
         if (ALG == ALG_SSSP && ROT && win) {

@@ -60,6 +60,7 @@ def main():
                 res = {}
                 for m in (A.MAP_THREAD, A.MAP_CTA):
                     p = A.policy_default(0)
+                    p.kind = A.POLICY_PAPER   # both forced variants in the same (general) kernel
                     p.mapping, p.workset = m, A.WS_QUEUE
                     st = run(G, alg, s, p, expect, trace=True)
                     res[m] = st

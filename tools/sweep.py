@@ -36,6 +36,8 @@ def variants(orders, kinds=(1,)):
                     out.append((name, dict(order=o, mapping=m, workset=w, kind=k)))
         out.append((f"{'O' if o else 'U'}_adaptive_paper", dict(order=o, kind=0)))
         out.append((f"{'O' if o else 'U'}_adaptive_tuned", dict(order=o, kind=1)))
+        if o:   # NEXT-3: the ordered bucket width adapted per iteration
+            out.append(("O_adaptive_tuned_delta0", dict(order=1, kind=1, delta=0)))
     return out
 
 
@@ -67,9 +69,9 @@ def main():
             if alg == "bfs" and kw.get("order") == 1 and False:
                 continue
             p = A.policy_default(0)
+            p.delta = args.delta
             for k, v in kw.items():
                 setattr(p, k, v)
-            p.delta = args.delta
             for k, v in extra.items():
                 setattr(p, k, int(v))
             times, edges, iters, traces, red = [], [], [], [], []
