@@ -104,8 +104,10 @@ typedef struct {
                                 iteration converts it to a queue in O(V/32) (the paper's update-vector bitmap,
                                 22.s13-14).  Used only on graphs without the degree layout (non-skewed; measured
                                 2x slower on R-MAT) unless free_ppm = 1000000 (every iteration, also on
-                                skewed graphs: a diagnostic / test setting).  BFS and ag_cc use t_free from this
-                                field, ag_sssp the same threshold.
+                                skewed graphs: a diagnostic / test setting) — except unordered BFS on a degree-layout
+                                graph, which the tuned policy runs in the general kernel specialisation (hybrid
+                                queue, no free output: measured faster there).  BFS and ag_cc use
+                                t_free from this field, ag_sssp the same threshold.
                                 0 = never; ag_policy_default: 3906 (V/256) */
     uint32_t small_ws;       /* tuned policy, graphs without hub lists: an iteration whose working set has fewer than
                                 small_ws elements runs on one CTA per SM while the others park (cheaper grid barrier;
@@ -131,7 +133,7 @@ typedef struct {
  * time so that the status words of high-degree vertices — the targets of most edges in a power-law
  * graph — are packed into a small, cache-resident prefix of the visited bitmap / state arrays.
  * Results are always returned in the caller's vertex ids.  AUTO picks DEGREE when the inspector
- * sees a skewed degree distribution (max_deg >= 64 x ceil(E/V)), else IDENTITY. */
+ * sees a skewed degree distribution (max_deg >= 64 x ceil(E/V)), else IDENTITY. DEGREE needs V < 2^31 (AG_ERR_UNSUPPORTED; AUTO then picks IDENTITY). */
 typedef enum { AG_LAYOUT_AUTO = 0, AG_LAYOUT_IDENTITY = 1, AG_LAYOUT_DEGREE = 2 } ag_layout;
 
 typedef struct {
@@ -244,7 +246,10 @@ ag_status ag_dist_init(int rank, int world, const void *nccl_unique_id128, int d
 ag_status ag_dist_free(ag_comm c);
 /* Owned vertex range of `rank` for a V-vertex graph partitioned over `world` ranks. */
 ag_status ag_dist_owned_range(uint32_t V, int rank, int world, uint32_t *begin, uint32_t *end);
-/* Every rank passes the SAME global CSR (host or device); each keeps its destination-owned part. */
+/* Every rank passes the SAME global CSR (host or device); each keeps its destination-owned part.  The
+ * global col_idx / weights are streamed through the device in 16M-entry chunks twice (count, then
+ * scatter), so a rank never holds the global graph, only its row offsets (8 (V+1) B) and its own part.
+ * Rows of the part keep their entries but not their order.  V < 2^31 (AG_ERR_UNSUPPORTED otherwise). */
 ag_status ag_dist_graph_load_csr(ag_comm c, uint32_t V, uint64_t E, const uint64_t *row_ptr,
                                  const uint32_t *col_idx, const uint32_t *weights, ag_graph *out_local);
 /* As above but every rank passes only ITS part: CSR rows over all V whose entries all have their

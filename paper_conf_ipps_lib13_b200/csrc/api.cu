@@ -804,7 +804,10 @@ ag_status ag_graph_load_csr_ex(uint32_t V, uint64_t E, const uint64_t *row_ptr, 
     if (layout == AG_LAYOUT_AUTO) {
         uint64_t avg = (E + V - 1) / V;
         layout = (E > 0 && (uint64_t)hs.max_deg >= 64ull * (avg ? avg : 1)) ? AG_LAYOUT_DEGREE : AG_LAYOUT_IDENTITY;
+        if (V >= 0x80000000u) layout = AG_LAYOUT_IDENTITY;   // the degree sort counts items in 31 bits
     }
+    if (layout == AG_LAYOUT_DEGREE && V >= 0x80000000u)
+        return lfail(set_error(AG_ERR_UNSUPPORTED, "the degree layout needs V < 2^31"));
     g->layout = layout;
     const bool deg = layout == AG_LAYOUT_DEGREE;
     // final arrays

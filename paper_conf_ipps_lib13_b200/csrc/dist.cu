@@ -144,44 +144,52 @@ using namespace ag;
 // kernels
 // ------------------------------------------------------------------------------------------------
 // count the owned entries of each row
-__global__ void dist_count_kernel(const uint64_t *rp, const uint32_t *col, uint32_t V, uint32_t b, uint32_t e,
-                                  uint64_t *cnt) {
-    const uint32_t lane = threadIdx.x & 31, warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
-    for (uint32_t u = warp; u < V; u += nwarps) {
-        uint64_t c = 0;
-        for (uint64_t k = rp[u] + lane; k < rp[u + 1]; k += 32) {
-            uint32_t v = col[k];
-            c += (v >= b && v < e);
-        }
-        c = warp_sum(c);
-        if (lane == 0) cnt[u] = c;
+// ---- partition extraction from a streamed global CSR (ag_dist_graph_load_csr): the global col_idx /
+// weights arrive in chunks; each pass handles the CSR entries [e0, e1) of one chunk, whose rows are
+// [ra, rb] (owner row of entry k: the largest u in [ra, rb] with rp[u] <= k).
+__device__ __forceinline__ uint32_t chunk_owner(const uint64_t *rp, uint32_t ra, uint32_t rb, uint64_t k) {
+    uint32_t lo = ra, hi = rb + 1;   // rp[lo] <= k < rp[hi]
+    while (hi - lo > 1) {
+        const uint32_t mid = lo + (hi - lo) / 2;
+        if (rp[mid] <= k) lo = mid; else hi = mid;
     }
-    if (blockIdx.x == 0 && threadIdx.x == 0) cnt[V] = 0;
+    return lo;
 }
 
-// scatter the owned entries (order within a row preserved by a warp ballot scan)
-__global__ void dist_scatter_kernel(const uint64_t *rp, const uint32_t *col, const uint32_t *w, uint32_t V,
-                                    uint32_t b, uint32_t e, const uint64_t *nrp, uint32_t *ncol, uint32_t *nw) {
-    const uint32_t lane = threadIdx.x & 31, warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
-    for (uint32_t u = warp; u < V; u += nwarps) {
-        uint64_t out = nrp[u];
-        for (uint64_t k0 = rp[u]; k0 < rp[u + 1]; k0 += 32) {
-            const uint64_t k = k0 + lane;
-            uint32_t v = 0;
-            bool keep = false;
-            if (k < rp[u + 1]) {
-                v = col[k];
-                keep = v >= b && v < e;
-            }
-            const unsigned m = __ballot_sync(0xffffffffu, keep);
-            if (keep) {
-                const uint64_t pos = out + __popc(m & ((1u << lane) - 1u));
-                ncol[pos] = v;
-                if (w) nw[pos] = w[k];
-            }
-            out += __popc(m);
+__global__ void dist_validate_rows_kernel(const uint64_t *rp, uint32_t V, uint64_t E, unsigned *bad) {
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < V; u += gridDim.x * blockDim.x)
+        if (rp[u + 1] < rp[u]) *bad = 1u;
+    if (blockIdx.x == 0 && threadIdx.x == 0 && (rp[0] != 0 || rp[V] != E)) *bad = 1u;
+}
+
+// pass 1: validate the chunk's entries (col < V, weight in [1, 2^31)) and count the owned ones per row
+__global__ void dist_chunk_count_kernel(const uint64_t *rp, uint32_t V, const uint32_t *colc, const uint32_t *wc,
+                                        uint64_t e0, uint64_t e1, uint32_t ra, uint32_t rb, uint32_t b, uint32_t e,
+                                        unsigned long long *cnt, unsigned *bad) {
+    unsigned bd = 0;
+    for (uint64_t k = e0 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < e1; k += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t c = colc[k - e0];
+        if (c >= V) bd |= 2u;
+        if (wc) {
+            const uint32_t x = wc[k - e0];
+            if (x == 0 || x >= 0x80000000u) bd |= 4u;
+        }
+        if (c >= b && c < e) atomicAdd(&cnt[chunk_owner(rp, ra, rb, k)], 1ull);
+    }
+    if (bd) atomicOr(bad, bd);
+}
+
+// pass 2: scatter the chunk's owned entries to their rows (order inside a row is not kept: rows need
+// not be sorted, include/agraph.h)
+__global__ void dist_chunk_scatter_kernel(const uint64_t *rp, const uint32_t *colc, const uint32_t *wc, uint64_t e0,
+                                          uint64_t e1, uint32_t ra, uint32_t rb, uint32_t b, uint32_t e,
+                                          unsigned long long *cursor, uint32_t *ncol, uint32_t *nw) {
+    for (uint64_t k = e0 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < e1; k += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t c = colc[k - e0];
+        if (c >= b && c < e) {
+            const unsigned long long pos = atomicAdd(&cursor[chunk_owner(rp, ra, rb, k)], 1ull);
+            ncol[pos] = c;
+            if (wc) nw[pos] = wc[k - e0];
         }
     }
 }
@@ -653,67 +661,113 @@ ag_status ag_dist_graph_load_csr(ag_comm c, uint32_t V, uint64_t E, const uint64
     if (!c || !out_local || !row_ptr || (!col_idx && E)) return set_error(AG_ERR_INVALID_ARG, "NULL argument");
     *out_local = nullptr;
     if (V == 0 || V >= 0xFFFFFFFFu) return set_error(AG_ERR_BAD_CSR, "V must be in [1, 2^32-1)");
+    if (V >= 0x80000000u) return set_error(AG_ERR_UNSUPPORTED, "ag_dist_graph_load_csr needs V < 2^31 (31-bit scan)");
     const int dev = c->device;
+    int sms = 0;
+    ag_status s = check_device(dev, &sms);
+    if (s != AG_OK) return s;
     cudaSetDevice(dev);
     uint32_t b, e;
     ag_dist_owned_range(V, c->rank, c->world, &b, &e);
-    // validate the global CSR by loading it (identity layout), then extract the owned part
-    ag_graph g0 = nullptr;
-    ag_status s = ag_graph_load_csr_ex(V, E, row_ptr, col_idx, weights, dev, AG_LAYOUT_IDENTITY, &g0);
-    if (s != AG_OK) return s;
-    // global row offsets as u64 (the store may have narrowed them)
-    uint64_t *rp64 = nullptr, *cnt = nullptr, *nrp = nullptr;
-    uint32_t *ncol = nullptr, *nw = nullptr;
-    const int grid = g0->num_sms * 8;
-    if ((s = dev_alloc((void **)&rp64, (size_t)(V + 1) * 8, dev)) != AG_OK) { ag_graph_free(g0); return s; }
-    cudaMemcpy(rp64, row_ptr, (size_t)(V + 1) * 8, cudaMemcpyDefault);
-    const uint32_t *gw = nullptr;
-    uint32_t *wtmp = nullptr;
-    if (weights) {  // the store keeps only interleaved (col,w); take the weights from the caller again
-        if ((s = dev_alloc((void **)&wtmp, E * 4 + 128, dev)) != AG_OK) { ag_graph_free(g0); dev_free(rp64, (size_t)(V + 1) * 8, dev); return s; }
-        cudaMemcpy(wtmp, weights, E * 4, cudaMemcpyDefault);
-        gw = wtmp;
-    }
+    // The global CSR is never held on the device: the row offsets are copied once, col_idx / weights
+    // stream through two chunk buffers twice — pass 1 validates and counts the owned entries per row,
+    // pass 2 scatters them — so device memory holds the row offsets, the chunk buffers and the owned
+    // part only (C5 / 8 ranks: ~3.5 GB instead of the ~34 GB of a staged global graph).
+    const uint64_t CH = 1ull << 24;
+    const size_t rpb = (size_t)(V + 1) * 8;
+    uint64_t *rp64 = nullptr, *rph = nullptr;
+    unsigned long long *cnt = nullptr, *nrp = nullptr;
+    uint32_t *colc = nullptr, *wc = nullptr, *ncol = nullptr, *nw = nullptr;
+    unsigned *bad = nullptr;
     void *tmp = nullptr;
     size_t tb = 0;
-    auto cleanup = [&]() {
-        dev_free(rp64, (size_t)(V + 1) * 8, dev);
-        dev_free(cnt, (size_t)(V + 1) * 8, dev);
-        dev_free(wtmp, E * 4 + 128, dev);
-        dev_free(tmp, tb, dev);
-        ag_graph_free(g0);
-    };
-    if ((s = dev_alloc((void **)&cnt, (size_t)(V + 1) * 8, dev)) != AG_OK) { cleanup(); return s; }
-    if ((s = dev_alloc((void **)&nrp, (size_t)(V + 1) * 8, dev)) != AG_OK) { cleanup(); return s; }
-    dist_count_kernel<<<grid, 256>>>(rp64, g0->d_col, V, b, e, cnt);
-    cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, nrp, (int)V + 1);
-    if ((s = dev_alloc(&tmp, tb, dev)) != AG_OK) { dev_free(nrp, (size_t)(V + 1) * 8, dev); cleanup(); return s; }
-    cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, nrp, (int)V + 1);
     uint64_t El = 0;
-    cudaMemcpy(&El, nrp + V, 8, cudaMemcpyDeviceToHost);
-    if ((s = dev_alloc((void **)&ncol, El * 4 + 128, dev)) != AG_OK) { dev_free(nrp, (size_t)(V + 1) * 8, dev); cleanup(); return s; }
-    if (gw && (s = dev_alloc((void **)&nw, El * 4 + 128, dev)) != AG_OK) {
-        dev_free(ncol, El * 4 + 128, dev);
-        dev_free(nrp, (size_t)(V + 1) * 8, dev);
-        cleanup();
-        return s;
-    }
-    dist_scatter_kernel<<<grid, 256>>>(rp64, g0->d_col, gw, V, b, e, nrp, ncol, nw);
-    note_launch(3);
-    cudaError_t ce = cudaDeviceSynchronize();
-    cleanup();
-    if (ce != cudaSuccess) {
+    auto cleanup = [&]() {
+        dev_free(rp64, rpb, dev);
+        dev_free(cnt, rpb, dev);
+        dev_free(nrp, rpb, dev);
+        dev_free(colc, CH * 4, dev);
+        dev_free(wc, CH * 4, dev);
         dev_free(ncol, El * 4 + 128, dev);
         dev_free(nw, El * 4 + 128, dev);
-        dev_free(nrp, (size_t)(V + 1) * 8, dev);
-        return cuda_status(ce, "dist partition");
+        dev_free(bad, 16, dev);
+        dev_free(tmp, tb, dev);
+        free(rph);
+    };
+    auto fail = [&](ag_status st) { cleanup(); return st; };
+    if ((s = dev_alloc((void **)&rp64, rpb, dev)) != AG_OK) return fail(s);
+    if ((s = dev_alloc((void **)&cnt, rpb, dev)) != AG_OK) return fail(s);
+    if ((s = dev_alloc((void **)&nrp, rpb, dev)) != AG_OK) return fail(s);
+    if ((s = dev_alloc((void **)&bad, 16, dev)) != AG_OK) return fail(s);
+    if (E && (s = dev_alloc((void **)&colc, CH * 4, dev)) != AG_OK) return fail(s);
+    if (E && weights && (s = dev_alloc((void **)&wc, CH * 4, dev)) != AG_OK) return fail(s);
+    rph = (uint64_t *)malloc(rpb);   // chunk -> row ranges are found on the host
+    if (!rph) return fail(set_error(AG_ERR_OOM, "host row_ptr copy"));
+    cudaError_t ce = cudaMemcpy(rph, row_ptr, rpb, cudaMemcpyDefault);
+    if (ce == cudaSuccess) ce = cudaMemcpy(rp64, rph, rpb, cudaMemcpyHostToDevice);
+    if (ce == cudaSuccess) ce = cudaMemset(bad, 0, 16);
+    if (ce == cudaSuccess) ce = cudaMemset(cnt, 0, rpb);
+    if (ce != cudaSuccess) return fail(cuda_status(ce, "dist partition"));
+    dist_validate_rows_kernel<<<sms * 4, 256>>>(rp64, V, E, bad);
+    note_launch(1);
+    unsigned hbad = 0;
+    ce = cudaMemcpy(&hbad, bad, 4, cudaMemcpyDeviceToHost);
+    if (ce != cudaSuccess) return fail(cuda_status(ce, "dist partition"));
+    if (hbad) return fail(set_error(AG_ERR_BAD_CSR, "invalid CSR (row offsets)"));
+    auto rows_of = [&](uint64_t e0, uint64_t e1, uint32_t &ra, uint32_t &rb) {   // rows touching [e0, e1)
+        uint32_t lo = 0, hi = V;   // ra: first u with rp[u+1] > e0
+        while (lo < hi) {
+            const uint32_t mid = lo + (hi - lo) / 2;
+            if (rph[mid + 1] > e0) hi = mid; else lo = mid + 1;
+        }
+        ra = lo;
+        lo = ra;
+        hi = V;   // rb: last u with rp[u] < e1
+        while (lo < hi) {
+            const uint32_t mid = lo + (hi - lo + 1) / 2;
+            if (rph[mid] < e1) lo = mid; else hi = mid - 1;
+        }
+        rb = lo;
+    };
+    for (int pass = 0; pass < 2; ++pass) {
+        if (pass == 1) {   // owned-entry offsets, then the owned part's arrays
+            cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, nrp, (int)V + 1);
+            if ((s = dev_alloc(&tmp, tb, dev)) != AG_OK) return fail(s);
+            cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, nrp, (int)V + 1);
+            ce = cudaMemcpy(&El, nrp + V, 8, cudaMemcpyDeviceToHost);
+            if (ce != cudaSuccess) return fail(cuda_status(ce, "dist partition"));
+            if ((s = dev_alloc((void **)&ncol, El * 4 + 128, dev)) != AG_OK) return fail(s);
+            if (weights && (s = dev_alloc((void **)&nw, El * 4 + 128, dev)) != AG_OK) return fail(s);
+            ce = cudaMemcpy(cnt, nrp, rpb, cudaMemcpyDeviceToDevice);   // cnt = per-row write cursor
+            if (ce != cudaSuccess) return fail(cuda_status(ce, "dist partition"));
+        }
+        for (uint64_t e0 = 0; e0 < E; e0 += CH) {
+            const uint64_t e1 = (E - e0 > CH) ? e0 + CH : E;
+            uint32_t ra, rb;
+            rows_of(e0, e1, ra, rb);
+            ce = cudaMemcpy(colc, col_idx + e0, (e1 - e0) * 4, cudaMemcpyDefault);
+            if (ce == cudaSuccess && weights) ce = cudaMemcpy(wc, weights + e0, (e1 - e0) * 4, cudaMemcpyDefault);
+            if (ce != cudaSuccess) return fail(cuda_status(ce, "dist partition copy"));
+            if (pass == 0)
+                dist_chunk_count_kernel<<<sms * 8, 256>>>(rp64, V, colc, weights ? wc : nullptr, e0, e1, ra, rb, b, e, cnt, bad);
+            else
+                dist_chunk_scatter_kernel<<<sms * 8, 256>>>(rp64, colc, weights ? wc : nullptr, e0, e1, ra, rb, b, e, cnt, ncol, nw);
+            note_launch(1);
+        }
+        if (pass == 0) {
+            ce = cudaMemcpy(&hbad, bad, 4, cudaMemcpyDeviceToHost);
+            if (ce != cudaSuccess) return fail(cuda_status(ce, "dist partition"));
+            if (hbad)
+                return fail(set_error(AG_ERR_BAD_CSR, "invalid CSR (%s%s)", hbad & 2 ? "col>=V " : "",
+                                      hbad & 4 ? "weight not in [1,2^31) " : ""));
+        }
     }
+    ce = cudaDeviceSynchronize();
+    if (ce != cudaSuccess) return fail(cuda_status(ce, "dist partition"));
     // the local part is an ordinary graph handle (rows over all V, owned destinations only)
     ag_graph gl = nullptr;
-    s = ag_graph_load_csr_ex(V, El, nrp, ncol, nw, dev, AG_LAYOUT_IDENTITY, &gl);
-    dev_free(ncol, El * 4 + 128, dev);
-    dev_free(nw, El * 4 + 128, dev);
-    dev_free(nrp, (size_t)(V + 1) * 8, dev);
+    s = ag_graph_load_csr_ex(V, El, (const uint64_t *)nrp, ncol, nw, dev, AG_LAYOUT_IDENTITY, &gl);
+    cleanup();
     if (s != AG_OK) return s;
     if ((s = part_alloc(gl, c)) != AG_OK) { ag_graph_free(gl); return s; }
     if (c->group) c->group->parts[c->rank] = gl;
