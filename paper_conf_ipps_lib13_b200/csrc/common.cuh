@@ -169,7 +169,7 @@ struct DevPolicy {
 //   * working set: the queue (appends are warp-staged, the bitmap scan costs O(V/32) per iteration),
 //     except the ordered-SSSP pending set once it holds >= V/32 vertices: a bucket then re-reads most
 //     of it, and one O(V/32) scan of the pending bitmap beats re-reading (and re-appending) the list;
-//   * mapping: THREAD for small working sets of low out-degree (m_F <= 16 |WS|) on graphs without
+//   * mapping: THREAD for small working sets of low out-degree (m_F <= 6 |WS|) on graphs without
 //     straggler lists (max degree <= 64), else HYBRID (load-balanced pieces + hub tasks).
 __host__ __device__ inline uint8_t select_variant(const DevPolicy &p, uint64_t ws, uint64_t ws_edges) {
     uint32_t map, wsr;
@@ -183,7 +183,7 @@ __host__ __device__ inline uint8_t select_variant(const DevPolicy &p, uint64_t w
         }
     } else {
         wsr = (p.ordered && ws >= ((uint64_t)p.V + 31) / 32) ? WS_BM : WS_QU;
-        const bool low_deg = ws_edges <= 16ull * ws;
+        const bool low_deg = ws_edges <= 6ull * ws;   // grid-like (avg 2-4); ER's 8 already prefers H (r02 sweep)
         map = (p.max_deg <= 64 && low_deg && ws < p.t2_tuned) ? MAP_T : MAP_H;
     }
     if (p.force_map) map = p.force_map;

@@ -80,6 +80,9 @@ struct TravArgs {
                                 // travels with the entry, hub tasks carry the entry index (nullptr: off)
 };
 
+#ifndef AG_HTILE
+#define AG_HTILE BS   // hybrid mapping: queue entries per tile at most (the tile's pieces still span the CTA)
+#endif
 #ifndef AG_BLIND
 #define AG_BLIND 1
 #endif
@@ -1217,7 +1220,8 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         uint32_t tile_n = BS;
         if (ws == WS_QU && map != MAP_T) {
             uint32_t want = (qn + 2 * nact - 1) / (2 * nact);
-            tile_n = want < 1u ? 1u : (want > (uint32_t)BS ? (uint32_t)BS : want);
+            const uint32_t cap = (map == MAP_H) ? (uint32_t)AG_HTILE : (uint32_t)BS;
+            tile_n = want < 1u ? 1u : (want > cap ? cap : want);
         }
         // entry slot of this thread: spread across warps for the warp mapping
         const uint32_t s_idx = (map == MAP_W || (map == MAP_B && a.pol.cta_group == 32))

@@ -124,13 +124,13 @@ def test_ag_select_tuned_rule(L):
     info.num_vertices, info.num_edges, info.max_deg = 1 << 20, 8 << 20, 40     # ER-like: max degree 40
     p = _tuned_policy()
     T, H, QU, BM = A.MAP_THREAD, A.MAP_HYBRID, A.WS_QUEUE, A.WS_BITMAP
-    assert A.select(p, info, 1000, 8000) == A.variant(T, QU)           # small, avg degree 8
-    assert A.select(p, info, 1000, 16000) == A.variant(T, QU)          # m_F = 16 |WS|: still low
-    assert A.select(p, info, 1000, 16001) == A.variant(H, QU)          # above: load-balanced
-    assert A.select(p, info, 65535, 8 * 65535) == A.variant(T, QU)
-    assert A.select(p, info, 65536, 8 * 65536) == A.variant(H, QU)     # big working set
+    assert A.select(p, info, 1000, 4000) == A.variant(T, QU)           # small, avg degree 4 (grid-like)
+    assert A.select(p, info, 1000, 6000) == A.variant(T, QU)           # m_F = 6 |WS|: still low
+    assert A.select(p, info, 1000, 6001) == A.variant(H, QU)           # above: load-balanced (ER's 8)
+    assert A.select(p, info, 65535, 4 * 65535) == A.variant(T, QU)
+    assert A.select(p, info, 65536, 4 * 65536) == A.variant(H, QU)     # big working set
     info.max_deg = 65                                                   # one long list: straggler risk
-    assert A.select(p, info, 1000, 8000) == A.variant(H, QU)
+    assert A.select(p, info, 1000, 4000) == A.variant(H, QU)
     # unordered: never the bitmap, however dense
     assert A.select(p, info, 1 << 20, 8 << 20) == A.variant(H, QU)
     # ordered SSSP pending set: bitmap from V/32 on
