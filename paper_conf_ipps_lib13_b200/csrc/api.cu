@@ -267,14 +267,16 @@ __global__ void reached_kernel(const uint32_t *out, const Off *rp, const uint32_
 // Exact overflow test after an SSSP traversal (enqueued behind it; returns at once unless a relaxation
 // exceeded MAX_FINITE): a reachable vertex left at INF behind a finite one.  Packed state in device ids.
 template <typename Off>
-__global__ void overflow_check_kernel(const Ctl *ctl, const unsigned long long *P, const Off *rp, const uint2 *cw, uint32_t V,
-                                      unsigned *sticky) {
+__global__ void overflow_check_kernel(const Ctl *ctl, const unsigned long long *P, bool packed, const Off *rp, const uint2 *cw,
+                                      uint32_t V, unsigned *sticky) {
     if (!*(volatile const unsigned *)&ctl->overflow) return;
+    // packed: (dist << 32) | parent words; else the distance-only u32 state (no parents requested)
+    auto dist = [&](uint32_t x) { return packed ? (uint32_t)(P[x] >> 32) : reinterpret_cast<const uint32_t *>(P)[x]; };
     bool bad = false;
     for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < V && !bad; u += gridDim.x * blockDim.x) {
-        if ((P[u] >> 32) == INF) continue;
+        if (dist(u) == INF) continue;
         for (Off e = rp[u]; e < rp[u + 1]; ++e)
-            if ((P[cw[e].x] >> 32) == INF) { bad = true; break; }
+            if (dist(cw[e].x) == INF) { bad = true; break; }
     }
     if (bad) atomicOr(sticky, 1u);
 }
@@ -405,6 +407,9 @@ ag_status check_policy(const ag_policy *p) {
 // ------------------------------------------------------------------------------------------------
 // traversal launch
 // ------------------------------------------------------------------------------------------------
+#ifndef AG_DONLY
+#define AG_DONLY 1
+#endif
 template <int ALG, int ORD, typename Off>
 static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t st) {
     // the tuned adaptive policy runs the specialisation without the paper's static variants
@@ -419,7 +424,12 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
                           (ALG == ALG_SSSP && ORD == ORD_O && a.pol.force_ws == WS_BM);
     const bool tuned = a.pol.kind == AG_POLICY_TUNED && tuned_map && tuned_ws &&
                        !(ALG == ALG_BFS && ORD == ORD_U && g->info.layout == AG_LAYOUT_DEGREE);
-    auto fn = tuned ? traverse_kernel<ALG, ORD, Off, true> : traverse_kernel<ALG, ORD, Off, false>;
+    // SSSP without parents in the tuned specialisation: distance-only state (u32)
+    const bool donly = AG_DONLY && ALG == ALG_SSSP && tuned && a.parent_out == nullptr;
+    g->last_packed = !donly;
+    auto fn = !tuned ? traverse_kernel<ALG, ORD, Off, false>
+              : donly ? traverse_kernel<ALG, ORD, Off, true, ALG == ALG_SSSP>
+                      : traverse_kernel<ALG, ORD, Off, true>;
     const size_t dyn = 0;
     if (dyn) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
     int occ = 0;
@@ -428,9 +438,10 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
     // L1/shared carveout: request just the shared memory the resident CTAs need so the rest of the
     // 256 KB goes to L1, where the status gathers hit (the driver otherwise picked a 132 KB shared
     // configuration for ~100 KB of use).  Once per kernel.
-    static int carved[2] = {0, 0};   // per specialisation (tuned / paper variants)
-    if (!carved[tuned]) {
-        carved[tuned] = 1;
+    static int carved[3] = {0, 0, 0};   // per specialisation (paper variants / tuned / tuned distance-only)
+    const int spec = tuned ? (donly ? 2 : 1) : 0;
+    if (!carved[spec]) {
+        carved[spec] = 1;
         int pct = -1;
         cudaFuncAttributes fa;
         if (cudaFuncGetAttributes(&fa, fn) == cudaSuccess) {
@@ -461,7 +472,7 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
     attrs[0].val.cooperative = 1;
     int nattr = 1;
     void *wbase = ALG == ALG_SSSP ? (void *)a.P : ALG == ALG_CC ? (void *)a.level : (void *)a.vis;
-    size_t wbytes = ALG == ALG_SSSP ? (size_t)g->V * 8 : ALG == ALG_CC ? (size_t)g->V * 4 : (size_t)g->nwords * 4;
+    size_t wbytes = ALG == ALG_SSSP ? (size_t)g->V * (donly ? 4 : 8) : ALG == ALG_CC ? (size_t)g->V * 4 : (size_t)g->nwords * 4;
     if (g->persist_bytes > 0) {
         if (wbytes > g->max_window) wbytes = g->max_window;
         attrs[1].id = cudaLaunchAttributeAccessPolicyWindow;
@@ -581,8 +592,8 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
     if (stats) cudaEventRecord(g->ev[1], st);
     if (alg == ALG_SSSP) {   // deferred exact overflow test (a no-op launch unless the traversal flagged one)
         Ctl *ctl = (Ctl *)g->d_ctl;
-        overflow_check_kernel<Off><<<g->num_sms * 4, 256, 0, st>>>(ctl, g->d_P, (const Off *)g->d_rp, g->d_cw, g->V,
-                                                                    &ctl->sticky);
+        overflow_check_kernel<Off><<<g->num_sms * 4, 256, 0, st>>>(ctl, g->d_P, g->last_packed, (const Off *)g->d_rp,
+                                                                    g->d_cw, g->V, &ctl->sticky);
         note_launch(1);
     }
     g->last_stream = st;

@@ -58,6 +58,7 @@ struct ag_graph_s {
     // deferred status: stream of the last enqueued traversal (the status itself is Ctl::sticky)
     cudaStream_t last_stream = nullptr;
     bool pending_check = false;
+    bool last_packed = true;       // the last SSSP kept the packed (dist, parent) state (false: distance-only u32)
     // multi-GPU
     ag_dist_part *dist = nullptr;
 };

@@ -102,7 +102,6 @@ struct __align__(16) TileSmem {
     uint32_t uval[BS];
     uint32_t deg[BS];
     uint32_t scan[BS + 1];
-    uint32_t wscan[BS + 1];
     uint32_t woff[2][WARPS_PER_CTA];
     uint32_t wq[WARPS_PER_CTA][WQ_CAP];   // per-warp staged queue appends (hybrid mapping)
     unsigned long long red64[2][WARPS_PER_CTA];
@@ -119,8 +118,12 @@ struct __align__(16) TileSmem {
 // Per-iteration operations of one algorithm (gate = which WS elements are expanded; visit = the
 // per-edge update).  Per-thread counters are reduced once per CTA at the end of the iteration.
 // ------------------------------------------------------------------------------------------------
-template <int ALG, int ORD, typename Off>
+// DO (SSSP, tuned kernels, no parents requested): the per-vertex state is the u32 distance alone (32-bit
+// atomicMin, 4-byte status gathers: half the L2/L1 footprint of the packed (dist, parent) word); the packed
+// 64-bit word is kept whenever parents are requested, so the parent stays consistent with its distance.
+template <int ALG, int ORD, typename Off, bool DO = false>
 struct Ops {
+    static_assert(!DO || ALG == ALG_SSSP, "distance-only state is an SSSP specialisation");
     static constexpr int EB = (ALG == ALG_SSSP) ? AG_EB_SSSP : AG_EB_BFS;
     const TravArgs<Off> &a;
     uint32_t it;
@@ -156,6 +159,22 @@ struct Ops {
         qlen_next = &a_.ctl->q_len[sn];
     }
 
+    // SSSP state accessors: distance of u (relaxed / status read), and the relaxation itself (returns the
+    // previous distance; the packed form also records the parent u in the same atomic)
+    __device__ __forceinline__ uint32_t *D() const { return reinterpret_cast<uint32_t *>(a.P); }
+    __device__ __forceinline__ uint32_t dist_now(uint32_t u) const {
+        if constexpr (DO) return ld_relaxed(D() + u);
+        else return (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
+    }
+    __device__ __forceinline__ uint32_t relax(uint32_t v, uint32_t nd, uint32_t u) const {
+        if constexpr (DO) return atomicMin(D() + v, nd);
+        else return (uint32_t)(atomicMin(&a.P[v], ((unsigned long long)nd << 32) | u) >> 32);
+    }
+    __device__ __forceinline__ void relax_red(uint32_t v, uint32_t nd, uint32_t u) const {
+        if constexpr (DO) red_min32(D() + v, nd);
+        else red_min64(&a.P[v], ((unsigned long long)nd << 32) | u);
+    }
+
     // Is working-set element u expanded in this iteration?  Fills its adjacency range and value.
     __device__ __forceinline__ bool gate(uint32_t u, Off &beg, uint32_t &deg, uint32_t &uval) {
         bool ex = true;
@@ -177,7 +196,7 @@ struct Ops {
         } else if (a.ulist) {
             // listed entry: uval (the sender's distance of u) was set by the caller; every entry expands
         } else {
-            uint32_t t = (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
+            uint32_t t = dist_now(u);
             uval = t;
             if constexpr (ORD == ORD_O) {
                 if ((uint64_t)t < hi) {  // in the current bucket: claim (settle) it
@@ -191,7 +210,7 @@ struct Ops {
                             // is visible after this fence: expand with the current value (the improver
                             // fences between its atomicMin and its atomicOr on the pending bit)
                             __threadfence();
-                            uval = (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
+                            uval = dist_now(u);
                         }
                     }
                 } else {  // pending survivor: stays in the working set, feeds findmin (22.s11)
@@ -240,7 +259,7 @@ struct Ops {
             u = key;
             uval = (ALG == ALG_BFS) ? it
                  : (ALG == ALG_CC)  ? ld_relaxed(&a.level[u])
-                                    : (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
+                                    : dist_now(u);
         }
     }
 
@@ -249,62 +268,10 @@ struct Ops {
     // read can only cause an extra atomic, never a missed update.
     using St = uint32_t;
     __device__ __forceinline__ St status(uint32_t v) const {
-        if constexpr (ALG == ALG_SSSP) return (uint32_t)(ld_keep(a.P + v, pol_keep) >> 32);
+        if constexpr (ALG == ALG_SSSP && DO) return ld_keep(D() + v, pol_keep);
+        else if constexpr (ALG == ALG_SSSP) return (uint32_t)(ld_keep(a.P + v, pol_keep) >> 32);
         else if constexpr (ALG == ALG_CC) return ld_keep(a.level + v, pol_keep);   // label[v]
         else return ld_keep(a.vis + (v >> 5), pol_keep);   // BFS: visited bit (level-synchronous: set <=> level <= current+1)
-    }
-
-    // Per-edge update for edge (u -> v, wt) from a frontier element with value uval, given status s.
-    // Returns true if v newly entered the next working set (the caller appends it to the queue).
-    __device__ __forceinline__ bool update(uint32_t u, uint32_t uval, uint32_t v, uint32_t wt, St s, bool valid) {
-        const uint32_t m = 1u << (v & 31);
-        bool nw = false;
-        if (!valid) return false;
-        if constexpr (ALG == ALG_CC) {
-            if (s > uval && atomicMin(&a.level[v], uval) > uval)          // m.label > n.label
-                nw = !(atomicOr(bm_next + (v >> 5), m) & m);               // ws.add(m), deduped
-        } else if constexpr (ALG == ALG_BFS) {
-            const uint32_t nl = uval + 1;
-            if constexpr (ORD == ORD_O) {
-                if (!(s & m)) {                                        // m.level == INF ?   (Fig. 4 l.8)
-                    if (!(atomicOr(a.vis + (v >> 5), m) & m)) {        // claim: first visit wins
-                        nw = true;
-                        a.level[v] = nl;                               // m.level = level    (l.9)
-                        if (a.parent) a.parent[v] = u;
-                        red_or(a.bm[(it + 1) % 3] + (v >> 5), m);      // update vector      (l.10)
-                    }
-                }
-            } else {
-                // m.level > level ?  (Fig. 4 l.8').  A set visited bit implies level[v] <= nl, so it is
-                // an exact pre-filter; the decision itself is the atomicMin on the level.
-                if (!(s & m)) {
-                    if (atomicMin(&a.level[v], nl) > nl) {
-                        nw = true;
-                        if (a.parent) a.parent[v] = u;
-                        red_or(a.vis + (v >> 5), m);
-                        red_or(bm_next + (v >> 5), m);
-                    }
-                }
-            }
-        } else {
-            const uint64_t nd = (uint64_t)uval + wt;                   // d = n.distance + w (Fig. 5 l.6)
-            if (nd > MAX_FINITE) {
-                ovf = true;
-            } else if ((uint64_t)s > nd) {                             // d < m.distance      (l.7)
-                unsigned long long old = atomicMin(&a.P[v], (nd << 32) | u);
-                if ((old >> 32) > nd) {                                // m.distance = d      (l.8)
-                    if (fenced) __threadfence();
-                    uint32_t ob = atomicOr(bm_next + (v >> 5), m);
-                    nw = !(ob & m);                                    // ws.add(m), deduped  (l.9)
-                    vmin = min(vmin, (uint32_t)nd);
-                    if constexpr (ORD == ORD_O) {
-                        if (nw) dpend += 1;
-                    }
-                }
-            }
-            if (ORD == ORD_O && !append_next) nw = false;
-        }
-        return nw;
     }
 
     // The updates of NB edges with their atomics phased: (1) candidates from the status words,
@@ -318,7 +285,7 @@ struct Ops {
         // (1) candidates from the (possibly stale) status words; CONV (all 32 lanes converged): a warp
         // with no candidate at all skips the atomic and resolution code (the common case on big levels)
         uint32_t cm = 0;   // bit j: an atomic is issued for edge j
-        uint64_t nd[NB];
+        uint32_t nd[NB];   // SSSP: candidate distance (<= MAX_FINITE whenever bit j of cm is set)
 #pragma unroll
         for (int j = 0; j < NB; ++j) {
             if constexpr (ALG == ALG_BFS) {
@@ -328,10 +295,11 @@ struct Ops {
                 nd[j] = uv[j];
                 if (ok[j] && st[j] > uv[j]) cm |= 1u << j;                      // m.label > n.label
             } else {
-                nd[j] = (uint64_t)uv[j] + wt[j];                                // d = n.distance + w (l.6)
+                const uint64_t d = (uint64_t)uv[j] + wt[j];                     // d = n.distance + w (l.6)
+                nd[j] = (uint32_t)d;
                 if (ok[j]) {
-                    if (nd[j] > MAX_FINITE) ovf = true;
-                    else if ((uint64_t)st[j] > nd[j]) cm |= 1u << j;            // d < m.distance      (l.7)
+                    if (d > MAX_FINITE) ovf = true;
+                    else if (st[j] > nd[j]) cm |= 1u << j;                      // d < m.distance      (l.7)
                 }
             }
         }
@@ -345,7 +313,7 @@ struct Ops {
             for (int j = 0; j < NB; ++j) {
                 if ((cm >> j) & 1u) {
                     if constexpr (ALG == ALG_SSSP) {
-                        red_min64(&a.P[v[j]], (nd[j] << 32) | u[j]);            // m.distance = d (l.8)
+                        relax_red(v[j], nd[j], u[j]);                           // m.distance = d (l.8)
                         vmin = min(vmin, (uint32_t)nd[j]);
                     } else if constexpr (ALG == ALG_CC) {
                         red_min32(&a.level[v[j]], uv[j]);                       // m.label = n.label
@@ -400,18 +368,18 @@ struct Ops {
                 }
             }
         } else {
-            unsigned long long r[NB];
+            uint32_t r[NB];   // previous distance of v[j]
 #pragma unroll
             for (int j = 0; j < NB; ++j) {
-                r[j] = 0ull;
-                if ((cm >> j) & 1u) r[j] = atomicMin(&a.P[v[j]], (nd[j] << 32) | u[j]);
+                r[j] = 0u;
+                if ((cm >> j) & 1u) r[j] = relax(v[j], nd[j], u[j]);
             }
             uint32_t ob[NB];
             uint32_t im = 0;   // bit j: we lowered m.distance
 #pragma unroll
             for (int j = 0; j < NB; ++j) {
                 ob[j] = 0u;
-                if (((cm >> j) & 1u) && (r[j] >> 32) > nd[j]) {         // m.distance = d      (l.8)
+                if (((cm >> j) & 1u) && r[j] > nd[j]) {                  // m.distance = d      (l.8)
                     if (fenced) __threadfence();
                     im |= 1u << j;
                     ob[j] = atomicOr(bm_next + (v[j] >> 5), 1u << (v[j] & 31));
@@ -522,43 +490,6 @@ struct Ops {
         batch_vals<N, true>(uu, vv, v, wt, ok);
     }
 
-    // One aligned window of WIN = 32 x EPL consecutive CSR entries [wbase, wbase + WIN), restricted to
-    // [lo, hi) (one adjacency list), processed by a whole warp: each lane issues ONE 16-byte vector
-    // load for its EPL entries, then EPL independent status loads, then the updates (all lanes
-    // converged; staged appends).  The per-edge owner lookup of the gather path disappears.
-    static constexpr int EPL = (ALG == ALG_SSSP) ? 2 : 4;
-    static constexpr int WIN = 32 * EPL;
-    __device__ __forceinline__ void window(uint32_t u, uint32_t uval, Off wbase, Off lo, Off hi) {
-        const Off e0 = wbase + (Off)lane_id() * EPL;
-        uint32_t v[EPL], wt[EPL];
-        bool ok[EPL];
-        const bool any = e0 < hi && e0 + EPL > lo;
-        if constexpr (ALG == ALG_SSSP) {
-            uint4 c = any ? ld_stream4(reinterpret_cast<const uint4 *>(a.cw + e0), pol_stream) : make_uint4(0, 1, 0, 1);
-            v[0] = c.x; wt[0] = c.y; v[1] = c.z; wt[1] = c.w;
-        } else {
-            uint4 c = any ? ld_stream4(reinterpret_cast<const uint4 *>(a.col + e0), pol_stream) : make_uint4(0, 0, 0, 0);
-            v[0] = c.x; v[1] = c.y; v[2] = c.z; v[3] = c.w;
-#pragma unroll
-            for (int j = 0; j < EPL; ++j) wt[j] = 1u;
-        }
-        St st[EPL];
-#pragma unroll
-        for (int j = 0; j < EPL; ++j) {
-            ok[j] = (e0 + j >= lo) && (e0 + j < hi);
-            st[j] = ok[j] ? status(v[j]) : (St)0;
-        }
-#pragma unroll
-        for (int j = 0; j < EPL; ++j) {
-            bool nw = update(u, uval, v[j], wt[j], st[j], ok[j]);
-            const unsigned m = __ballot_sync(0xffffffffu, nw);
-            if (nw) wbuf[wfill + __popc(m & ((1u << lane_id()) - 1u))] = v[j];
-            wfill += __popc(m);
-        }
-        __syncwarp();
-        if (wfill >= 32) warp_flush(false);
-    }
-
     // Copy this warp's staged entries (all, or whole groups of 32) to the global queue.
     __device__ __forceinline__ void warp_flush(bool all) {
         const unsigned lane = lane_id();
@@ -608,8 +539,8 @@ struct Ops {
 };
 
 // ------------------------------------------------------------------------------------------------
-template <int ALG, int ORD, typename Off, typename SmT>
-__device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, SmT &sm, Ctl *ctl,
+template <int ALG, int ORD, typename Off, bool DO, typename SmT>
+__device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off, DO> &ops, SmT &sm, Ctl *ctl,
                                                    uint32_t slot) {
     const unsigned lane = lane_id(), wid = threadIdx.x >> 5;
     unsigned long long ne = warp_sum(ops.ne), nv = warp_sum(ops.nv);
@@ -664,8 +595,8 @@ __device__ __forceinline__ void block_reduce_flush(Ops<ALG, ORD, Off> &ops, SmT 
 // ------------------------------------------------------------------------------------------------
 // One tile: thread tid holds working-set element (valid, u).  Applies the mapping.
 // ------------------------------------------------------------------------------------------------
-template <bool TUNED, int ALG, int ORD, typename Off, typename SmT>
-__device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off> &ops, SmT &sm, uint32_t map,
+template <bool TUNED, int ALG, int ORD, typename Off, bool DO, typename SmT>
+__device__ __forceinline__ void process_tile(Ops<ALG, ORD, Off, DO> &ops, SmT &sm, uint32_t map,
                                              bool valid, uint32_t u, uint32_t group, bool hubs, uint32_t slot,
                                              uint32_t uval_in = 0, uint32_t key = 0xFFFFFFFFu) {
     const TravArgs<Off> &a = ops.a;
@@ -804,8 +735,8 @@ __device__ __forceinline__ unsigned long long hub_wait(const TravArgs<Off> &a, u
 // drain the hub-chunk tasks of this iteration (hybrid mapping).  Thread 0 runs two claims ahead and
 // loads the next task word before the CTA expands the current one, so in steady state the claim and
 // fetch latency hides behind the expansion; tasks reach the CTA through two shared-memory slots.
-template <int ALG, int ORD, typename Off, typename SmT>
-__device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off> &ops, SmT &sm, uint32_t slot) {
+template <int ALG, int ORD, typename Off, bool DO, typename SmT>
+__device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off, DO> &ops, SmT &sm, uint32_t slot) {
     const TravArgs<Off> &a = ops.a;
     Ctl *ctl = a.ctl;
     __syncthreads();
@@ -975,7 +906,7 @@ __device__ __forceinline__ void compact_bitmap(const uint32_t *bm, uint32_t nwor
 // ------------------------------------------------------------------------------------------------
 // TUNED = the adaptive B200 policy only (thread / hybrid mappings over the queue): the paper's
 // static variants are compiled out, which frees registers for occupancy.
-template <int ALG, int ORD, typename Off, bool TUNED>
+template <int ALG, int ORD, typename Off, bool TUNED, bool DO = false>
 __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T : AG_MINB_SSSP)
                                                       : (TUNED ? AG_MINB_BFS_T : AG_MINB_BFS))
     traverse_kernel(const TravArgs<Off> a) {
@@ -997,6 +928,9 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             a.level[v] = a.perm ? a.perm[v] : v;
             a.q[0][v] = v;
         }
+    } else if (DO) {
+        uint32_t *D = reinterpret_cast<uint32_t *>(a.P);
+        for (uint32_t v = gtid; v < a.V; v += gthreads) D[v] = (v == src) ? 0u : INF;
     } else {
         for (uint32_t v = gtid; v < a.V; v += gthreads)
             a.P[v] = (v == src) ? (unsigned long long)src : INF64;   // dist 0, parent src
@@ -1200,7 +1134,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
             }
         }
 
-        Ops<ALG, ORD, Off> ops(a, it, hi, append);
+        Ops<ALG, ORD, Off, DO> ops(a, it, hi, append);
         ops.wbuf = sm.wq[threadIdx.x >> 5];
         ops.nact = nact;
         ops.bm_upd = !(TUNED && ALG == ALG_BFS);
@@ -1308,7 +1242,10 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     // exact overflow test (rare path: only when a relaxation exceeded MAX_FINITE): a reachable vertex
     // left at INF behind a finite one.  The packed state is final here (every CTA passed the barrier
     // that ended the last iteration, or was parked without writing), so no further barrier is needed.
-    if (ALG == ALG_SSSP) {  // unpack (dist, parent) into the caller's arrays (caller ids)
+    if (ALG == ALG_SSSP && DO) {  // distances into the caller's array (caller ids)
+        const uint32_t *D = reinterpret_cast<const uint32_t *>(a.P);
+        for (uint32_t v = gtid; v < a.V; v += gthreads) a.dist_out[v] = D[a.inv ? a.inv[v] : v];
+    } else if (ALG == ALG_SSSP) {  // unpack (dist, parent) into the caller's arrays (caller ids)
         for (uint32_t v = gtid; v < a.V; v += gthreads) {
             unsigned long long pv = a.P[a.inv ? a.inv[v] : v];
             a.dist_out[v] = (uint32_t)(pv >> 32);

@@ -89,6 +89,11 @@ def check_sssp(g, G, s, p, expect_dist=None):
         assert st.iterations == oracle.ordered_sssp_iterations(d)
     else:
         assert st.vertices_expanded >= Vr and st.edges_inspected >= Er
+    # no parents requested: the tuned kernels keep the distance-only u32 state instead of the packed word
+    out2, _, st2 = G.sssp(s, policy=p, stats=True)
+    assert np.array_equal(out2, d), f"SSSP dist (no parents) differ ({pname(p)}, src {s}): " \
+        f"{np.count_nonzero(out2 != d)} mismatches"
+    assert (st2.reached, st2.reached_edges) == (Vr, Er)
     return st
 
 
@@ -506,6 +511,15 @@ def test_deferred_overflow_is_sticky_across_queries():
     with pytest.raises(A.AgError) as e:           # the earlier overflow survives the later good query
         G.check()
     assert e.value.status == "AG_ERR_OVERFLOW"
+    # the same with parents requested (packed (dist, parent) state instead of the distance-only one)
+    par = torch.empty(g.V, dtype=torch.int32, device="cuda")
+    G.sssp(0, dist=out, parents=par, stream=stream)
+    G.sssp(1, dist=out, parents=par, stream=stream)
+    with pytest.raises(A.AgError) as e:
+        G.check()
+    assert e.value.status == "AG_ERR_OVERFLOW"
+    G.sssp(1, dist=out, parents=par, stream=stream)
+    G.check()
 
 
 @pytest.mark.parametrize("mode", ["window", "delta"])
