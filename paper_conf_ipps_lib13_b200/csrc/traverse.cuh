@@ -732,26 +732,26 @@ __device__ __forceinline__ unsigned long long hub_wait(const TravArgs<Off> &a, u
     }
 }
 
-// drain the hub-chunk tasks of this iteration (hybrid mapping).  Thread 0 runs two claims ahead and
-// loads the next task word before the CTA expands the current one, so in steady state the claim and
-// fetch latency hides behind the expansion; tasks reach the CTA through two shared-memory slots.
+// drain the hub-chunk tasks of this iteration (hybrid mapping).  Thread 0 claims the next task when the
+// current one starts and loads its word while the CTA expands the current one, so in steady state the
+// claim and fetch latency hides behind the expansion; tasks reach the CTA through two shared-memory slots.
 template <int ALG, int ORD, typename Off, bool DO, typename SmT>
 __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off, DO> &ops, SmT &sm, uint32_t slot) {
     const TravArgs<Off> &a = ops.a;
     Ctl *ctl = a.ctl;
     __syncthreads();
-    uint32_t c1 = 0, c2 = 0;          // claimed task indices: next, and the one after
-    unsigned long long pre = 0ull;    // prefetched word of task c1
+    // ONE task claimed ahead of the one being expanded (two ahead left up to two claimed-but-unstarted tasks
+    // per CTA when the ring ran dry, a tail of up to two tasks: C2 BFS -2.6%, SSSP -2.4% with one, A/B 11)
+    uint32_t c1 = 0;                  // claimed index of the next task
+    unsigned long long pre = 0ull;    // its word, fetched while the current task is expanded
     if (threadIdx.x == 0) {
         __threadfence();
         atomicAdd(&ctl->stage_done[slot], 1u);
         const uint32_t c0 = atomicAdd(&ctl->hub_head[slot], 1u);
-        c1 = atomicAdd(&ctl->hub_head[slot], 1u);
         const unsigned long long w = hub_wait(a, c0, slot, ops.nact);
         if (w) {
             a.hub[c0] = 0ull;
-            pre = c1 < a.hub_cap ? ld_relaxed64(a.hub + c1) : 0ull;
-            c2 = atomicAdd(&ctl->hub_head[slot], 1u);
+            c1 = atomicAdd(&ctl->hub_head[slot], 1u);
         }
         sm.htask[0] = w;
     }
@@ -769,6 +769,8 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off, DO> &ops, SmT &sm,
         constexpr uint32_t QE = Ops<ALG, ORD, Off>::QE;
         constexpr int QB = Ops<ALG, ORD, Off>::QB;
         const Off q0 = b / QE, q1 = (e + QE - 1) / QE;
+        // the next task was claimed before this one started; its word is fetched now, behind the expansion
+        if (threadIdx.x == 0) pre = c1 < a.hub_cap ? ld_relaxed64(a.hub + c1) : 0ull;
         for (Off qb = q0; qb < q1; qb += (Off)QB * BS) {
             uint32_t pu[QB], pv[QB];
             Off pq[QB], plo[QB], phi[QB];
@@ -788,9 +790,7 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off, DO> &ops, SmT &sm,
             const unsigned long long wn = pre ? pre : hub_wait(a, c1, slot, ops.nact);
             if (wn) {
                 a.hub[c1] = 0ull;
-                c1 = c2;
-                pre = c1 < a.hub_cap ? ld_relaxed64(a.hub + c1) : 0ull;
-                c2 = atomicAdd(&ctl->hub_head[slot], 1u);
+                c1 = atomicAdd(&ctl->hub_head[slot], 1u);
             }
             sm.htask[par ^ 1] = wn;
         }
@@ -1239,15 +1239,16 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         if (ab) atomicMax(&ctl->sticky, ab << 8);
         ctl->launch_seq += 1u;   // every CTA read it before the first grid barrier
     }
-    // exact overflow test (rare path: only when a relaxation exceeded MAX_FINITE): a reachable vertex
-    // left at INF behind a finite one.  The packed state is final here (every CTA passed the barrier
-    // that ended the last iteration, or was parked without writing), so no further barrier is needed.
+    // final pass: results into the caller's arrays in caller ids.  The state is final here (every CTA passed
+    // the barrier that ended the last iteration, or was parked without writing), so no further barrier is
+    // needed.  (The exact overflow test is a separate kernel, api.cu overflow_check_kernel.)
     if (ALG == ALG_SSSP && DO) {  // distances into the caller's array (caller ids)
+        // (a gather per output: measured 1-3% faster than coalesced reads with scattered stores, A/B 10)
         const uint32_t *D = reinterpret_cast<const uint32_t *>(a.P);
         for (uint32_t v = gtid; v < a.V; v += gthreads) a.dist_out[v] = D[a.inv ? a.inv[v] : v];
     } else if (ALG == ALG_SSSP) {  // unpack (dist, parent) into the caller's arrays (caller ids)
         for (uint32_t v = gtid; v < a.V; v += gthreads) {
-            unsigned long long pv = a.P[a.inv ? a.inv[v] : v];
+            const unsigned long long pv = a.P[a.inv ? a.inv[v] : v];
             a.dist_out[v] = (uint32_t)(pv >> 32);
             if (a.parent_out) {
                 uint32_t pp = (uint32_t)pv;

@@ -1,7 +1,8 @@
 #!/usr/bin/env python
 """Build experiment variants of libagraph.so into exp_libs/ (A/B on the GPU with tools/cmp_libs.sh).
 
-    python tools/mk_exp_libs.py NAME=DEF1,DEF2 NAME2= ...      (empty define list = the default build)
+    python tools/mk_exp_libs.py [--keep] NAME=DEF1,DEF2 NAME2= ...   (empty define list = the default build;
+                                                                   --keep: do not clear exp_libs/ first)
 """
 import os
 import sys
@@ -21,8 +22,10 @@ def one(spec):
 
 if __name__ == "__main__":
     os.makedirs(os.path.join(ROOT, "exp_libs"), exist_ok=True)
-    for f in os.listdir(os.path.join(ROOT, "exp_libs")):
-        os.remove(os.path.join(ROOT, "exp_libs", f))
-    with ThreadPoolExecutor(len(sys.argv) - 1) as ex:
-        for o in ex.map(one, sys.argv[1:]):
+    specs = [a for a in sys.argv[1:] if a != "--keep"]
+    if "--keep" not in sys.argv:
+        for f in os.listdir(os.path.join(ROOT, "exp_libs")):
+            os.remove(os.path.join(ROOT, "exp_libs", f))
+    with ThreadPoolExecutor(len(specs)) as ex:
+        for o in ex.map(one, specs):
             print(o)
