@@ -384,7 +384,7 @@ DevPolicy resolve_policy(const ag_policy &p, const ag_graph_s &g) {
     // arrivals instead of ~740 (measured C3 grid: BFS 55.9 -> 42.4 ms, SSSP 129 -> 92.7 ms with 148 CTAs)
     d.small_ctas = (uint32_t)g.num_sms;
     d.t_small = p.kind == AG_POLICY_TUNED ? (p.small_ws ? p.small_ws : 32768u) : 0u;
-    d.t_small_hub = p.kind == AG_POLICY_TUNED ? 4096u : 0u;   // C2: BFS -1.6%, SSSP -2.7% (median of 12)
+    d.t_small_hub = p.kind == AG_POLICY_TUNED ? (uint32_t)AG_T_SMALL_HUB : 0u;   // C2: BFS -1.6%, SSSP -2.7% (median of 12)
     d.smallchunk_per_cta = SMALLCHUNK_PER_CTA;
     d.ordered = p.order == AG_ORDERED ? 1u : 0u;
     // NEXT-3: the SSSP order axis adapted per iteration from the measured redundancy
@@ -423,7 +423,7 @@ static ag_status launch_traverse(ag_graph_s *g, TravArgs<Off> &a, cudaStream_t s
     const bool tuned_ws = a.pol.force_ws == 0 || a.pol.force_ws == WS_QU ||
                           (ALG == ALG_SSSP && ORD == ORD_O && a.pol.force_ws == WS_BM);
     const bool tuned = a.pol.kind == AG_POLICY_TUNED && tuned_map && tuned_ws &&
-                       !(ALG == ALG_BFS && ORD == ORD_U && g->info.layout == AG_LAYOUT_DEGREE);
+                       !(AG_BFS_ROUTE && ALG == ALG_BFS && ORD == ORD_U && g->info.layout == AG_LAYOUT_DEGREE);
     // SSSP without parents in the tuned specialisation: distance-only state (u32)
     const bool donly = AG_DONLY && ALG == ALG_SSSP && tuned && a.parent_out == nullptr;
     g->last_packed = !donly;

@@ -81,6 +81,14 @@ constexpr uint32_t HUB_CHUNK = AG_HUBCHUNK;
 #endif
 constexpr uint32_t HUB_CHUNK_SMALL = AG_HUBCHUNK_SMALL;
 constexpr uint32_t SMALLCHUNK_PER_CTA = AG_SMALLCHUNK_PER_CTA;
+// small-frontier mode on graphs with hub tasks: only in the falling tail, below this |WS|
+#ifndef AG_T_SMALL_HUB
+#define AG_T_SMALL_HUB 4096
+#endif
+// unordered BFS on degree-layout graphs runs the general specialisation with the tuned decisions
+#ifndef AG_BFS_ROUTE
+#define AG_BFS_ROUTE 1
+#endif
 // Edges processed per thread per batch: loads of all EB edges are issued before any dependent use.
 constexpr int EB_MAX = (AG_EB_BFS > AG_EB_SSSP) ? AG_EB_BFS : AG_EB_SSSP;
 

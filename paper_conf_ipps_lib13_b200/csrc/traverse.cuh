@@ -37,7 +37,8 @@ namespace ag {
 // diagnostic build only: per (iteration, CTA) timestamps — iteration start, tile loop done, hub drain
 // done — read back with ag_debug_prof() (tools/prof_iters.py)
 constexpr int PROF_IT = 64, PROF_CTA = 2048;
-__device__ unsigned long long g_prof[PROF_IT][PROF_CTA][4];   // [3]: adjacency entries gated by the CTA's tiles
+__device__ unsigned long long g_prof[PROF_IT][PROF_CTA][6];   // [3]: adjacency entries gated by the CTA's tiles,
+                                                               // [4]: hub tasks it expanded, [5]: when its first task arrived
 #define AG_PROF_MARK(it, k) \
     if (threadIdx.x == 0 && (it) < PROF_IT && blockIdx.x < PROF_CTA) g_prof[it][blockIdx.x][k] = globaltimer_ns()
 #else
@@ -754,6 +755,12 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off, DO> &ops, SmT &sm,
             c1 = atomicAdd(&ctl->hub_head[slot], 1u);
         }
         sm.htask[0] = w;
+#ifdef AG_PROF
+        if (ops.it < PROF_IT && blockIdx.x < PROF_CTA) {
+            g_prof[ops.it][blockIdx.x][4] = 0;
+            g_prof[ops.it][blockIdx.x][5] = w ? globaltimer_ns() : 0ull;
+        }
+#endif
     }
     __syncthreads();
     int par = 0;
@@ -786,6 +793,9 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off, DO> &ops, SmT &sm,
             }
             ops.template pieces<QB>(pu, pv, pq, plo, phi, pok);
         }
+#ifdef AG_PROF
+        if (threadIdx.x == 0 && ops.it < PROF_IT && blockIdx.x < PROF_CTA) g_prof[ops.it][blockIdx.x][4] += 1;
+#endif
         if (threadIdx.x == 0) {
             const unsigned long long wn = pre ? pre : hub_wait(a, c1, slot, ops.nact);
             if (wn) {

@@ -36,7 +36,7 @@ def main():
     fn = G.bfs if args.alg == "bfs" else G.sssp
     for _ in range(2):
         _, _, st = fn(src, stats=True, trace_cap=256)
-    buf = np.zeros((PROF_IT, PROF_CTA, 4), dtype=np.uint64)
+    buf = np.zeros((PROF_IT, PROF_CTA, 6), dtype=np.uint64)
     L = A.lib()
     L.ag_debug_prof.restype = ctypes.c_int
     L.ag_debug_prof.argtypes = [ctypes.c_void_p, ctypes.c_size_t]
@@ -45,7 +45,8 @@ def main():
     nb = int((buf[0, :, 0] > 0).sum())
     print(f"{args.config} {args.alg} src={src} ms={st.device_ms:.3f} iters={st.iterations} ctas={nb}")
     print(" it      |WS|   start->tiles done (first/med/last)   drains done (first/med/last)   next start"
-          "   gated edges: slowest-tile CTA / max / median")
+          "   gated edges: slowest-tile CTA / max / median   hub tasks per CTA: min / med / max (last CTA)"
+          "   first task at: min / med / max")
     for it in range(min(st.iterations, PROF_IT)):
         b = buf[it, :nb].astype(np.int64)
         t0 = b[:, 0].min()
@@ -54,7 +55,10 @@ def main():
         ws = int(st.trace_ws[it]) if it < len(st.trace_ws) else -1
         print(f"{it:3d} {ws:9d}   {tiles.min():7.1f} {np.median(tiles):7.1f} {tiles.max():7.1f}        "
               f"{drain.min():7.1f} {np.median(drain):7.1f} {drain.max():7.1f}       {nxt:7.1f}"
-              f"   {int(b[np.argmax(tiles), 3]):9d} {int(b[:, 3].max()):9d} {int(np.median(b[:, 3])):9d}")
+              f"   {int(b[np.argmax(tiles), 3]):9d} {int(b[:, 3].max()):9d} {int(np.median(b[:, 3])):9d}"
+              f"   {int(b[:, 4].min()):4d} {int(np.median(b[:, 4])):4d} {int(b[:, 4].max()):4d} ({int(b[np.argmax(drain), 4]):4d})"
+              + (lambda f: f"   {f.min():7.1f} {np.median(f):7.1f} {f.max():7.1f}" if f.size else "   -")(
+                  (b[b[:, 5] > 0, 5] - t0) / 1e3))
 
 
 if __name__ == "__main__":
