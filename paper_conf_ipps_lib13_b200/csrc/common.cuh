@@ -98,6 +98,14 @@ constexpr int EB_MAX = (AG_EB_BFS > AG_EB_SSSP) ? AG_EB_BFS : AG_EB_SSSP;
 // slot(it+2) is reset at the start of iteration it (its last reader finished at the barrier).
 // ---------------------------------------------------------------------------------------------
 constexpr int NGRP = 32;            // barrier arrival groups (hierarchical arrival)
+#ifndef AG_CTL_SPREAD
+#define AG_CTL_SPREAD 1
+#endif
+#if AG_CTL_SPREAD
+#define AG_CTL_LINE alignas(128)
+#else
+#define AG_CTL_LINE
+#endif
 
 struct alignas(128) Ctl {
     unsigned long long bar_word;      // (generation << 32) | payload, released by the last arriver
@@ -105,13 +113,17 @@ struct alignas(128) Ctl {
     unsigned int bar_count;           // groups arrived
     unsigned int pad1[31];
     unsigned int grp_count[NGRP * 32];  // CTAs arrived per group (one 128-B line each)
-    unsigned int q_len[3];            // queue append cursor == |WS| for BFS and unordered SSSP
-    unsigned int next_min[3];         // ordered SSSP: min tentative distance of pending vertices
-    unsigned int tile_ctr[3];         // dynamic tile scheduler
-    unsigned int hub_tail[3];         // hybrid mapping: produced hub-chunk tasks
-    unsigned int hub_head[3];         //                 consumed hub-chunk tasks
-    unsigned int stage_done[3];       //                 CTAs done producing
-    unsigned long long it_edges[3];   // edges inspected in iteration (m_F: selector input, trace)
+    // The counters every CTA hits with atomics or polls each iteration, one 128-B line each: an L2 slice
+    // serialises the operations on one line, and with the counters packed into two lines the queue appends,
+    // tile claims, hub claims, the drain's polls and the per-CTA reductions all queued behind each other
+    // (C2 BFS -3.5%, SSSP -6.6%, profiles/r02_ab/ab_summary.txt item 5p)
+    AG_CTL_LINE unsigned int q_len[3];       // queue append cursor == |WS| for BFS and unordered SSSP
+    AG_CTL_LINE unsigned int next_min[3];    // ordered SSSP: min tentative distance of pending vertices
+    AG_CTL_LINE unsigned int tile_ctr[3];    // dynamic tile scheduler
+    AG_CTL_LINE unsigned int hub_tail[3];    // hybrid mapping: produced hub-chunk tasks
+    AG_CTL_LINE unsigned int hub_head[3];    //                 consumed hub-chunk tasks
+    AG_CTL_LINE unsigned int stage_done[3];  //                 CTAs done producing
+    AG_CTL_LINE unsigned long long it_edges[3];   // edges inspected in iteration (m_F: selector input, trace)
     unsigned long long it_nv[3];      // working-set elements expanded in iteration
     unsigned int it_reexp[3];         // SSSP: expansions of a vertex already expanded earlier in the query
     unsigned int free_any[3];         // free-output iteration wrote at least one next-bitmap bit
