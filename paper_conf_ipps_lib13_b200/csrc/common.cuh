@@ -124,14 +124,14 @@ struct alignas(128) Ctl {
     AG_CTL_LINE unsigned int hub_head[3];    //                 consumed hub-chunk tasks
     AG_CTL_LINE unsigned int stage_done[3];  //                 CTAs done producing
     AG_CTL_LINE unsigned long long it_edges[3];   // edges inspected in iteration (m_F: selector input, trace)
-    unsigned long long it_nv[3];      // working-set elements expanded in iteration
-    unsigned int it_reexp[3];         // SSSP: expansions of a vertex already expanded earlier in the query
-    unsigned int free_any[3];         // free-output iteration wrote at least one next-bitmap bit
-    unsigned int pend_count;          // ordered SSSP: |pending|
-    unsigned int overflow;            // a relaxation exceeded MAX_FINITE
+    AG_CTL_LINE unsigned long long it_nv[3];      // working-set elements expanded in iteration
+    AG_CTL_LINE unsigned int it_reexp[3];         // SSSP: expansions of a vertex already expanded earlier in the query
+    AG_CTL_LINE unsigned int free_any[3];         // free-output iteration wrote at least one next-bitmap bit
+    AG_CTL_LINE unsigned int pend_count;          // ordered SSSP: |pending|
+    AG_CTL_LINE unsigned int overflow;            // a relaxation exceeded MAX_FINITE
     unsigned int iterations;
     unsigned int aborted;             // iteration cap hit (never expected)
-    unsigned long long vexp, eexp;    // totals
+    AG_CTL_LINE unsigned long long vexp, eexp;    // totals (adjacent: cleared together)
     // small-frontier mode (tuned kernels): CTAs >= small_ctas park while |WS| < t_small and are woken
     // with the iteration to resume at (wake_n = 0: terminate).  Own 128-B line: the parked CTAs poll
     // it, and must not slow the atomics on the per-iteration counters above.
