@@ -407,9 +407,6 @@ ag_status check_policy(const ag_policy *p) {
 // ------------------------------------------------------------------------------------------------
 // traversal launch
 // ------------------------------------------------------------------------------------------------
-#ifndef AG_LVL_SWZ
-#define AG_LVL_SWZ 1
-#endif
 #ifndef AG_DONLY
 #define AG_DONLY 1
 #endif
@@ -548,11 +545,10 @@ static ag_status run_query(ag_graph_s *g, int alg, uint32_t src, uint32_t *out, 
     a.inv = g->d_inv;
     if (alg != ALG_SSSP) {   // BFS levels / CC labels
         if (g->d_inv) {  // traverse in the degree layout, gather back to caller ids at the end
-            if (!g->d_level && (s = dev_alloc((void **)&g->d_level, level_bytes(g->V), g->device)) != AG_OK) return s;
+            if (!g->d_level && (s = dev_alloc((void **)&g->d_level, (size_t)g->V * 4 + 128, g->device)) != AG_OK) return s;
             if (d_par && !g->d_lpar && (s = dev_alloc((void **)&g->d_lpar, (size_t)g->V * 4 + 128, g->device)) != AG_OK)
                 return s;
             a.level = g->d_level;
-            a.lvl_swz = (alg == ALG_BFS && AG_LVL_SWZ) ? 1u : 0u;
             a.parent = d_par ? g->d_lpar : nullptr;
             a.out_level = d_out;
             a.out_parent = d_par;
@@ -975,7 +971,7 @@ ag_status ag_graph_free(ag_graph g) {
     dev_free(g->d_trace, g->trace_bytes, g->device);
     dev_free(g->d_perm, V * 4, g->device);
     dev_free(g->d_inv, V * 4, g->device);
-    dev_free(g->d_level, level_bytes(g->V), g->device);
+    dev_free(g->d_level, V * 4 + 128, g->device);
     dev_free(g->d_lpar, V * 4 + 128, g->device);
     if (g->ev[0]) cudaEventDestroy(g->ev[0]);
     if (g->ev[1]) cudaEventDestroy(g->ev[1]);

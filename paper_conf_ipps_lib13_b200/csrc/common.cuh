@@ -131,7 +131,8 @@ struct alignas(128) Ctl {
     AG_CTL_LINE unsigned int overflow;            // a relaxation exceeded MAX_FINITE
     unsigned int iterations;
     unsigned int aborted;             // iteration cap hit (never expected)
-    AG_CTL_LINE unsigned long long vexp, eexp;    // totals (adjacent: cleared together)
+    AG_CTL_LINE unsigned long long vexp;   // totals (adjacent: cleared together; ONE declarator per alignas,
+    unsigned long long eexp;               // which would otherwise align each of them)
     // small-frontier mode (tuned kernels): CTAs >= small_ctas park while |WS| < t_small and are woken
     // with the iteration to resume at (wake_n = 0: terminate).  Own 128-B line: the parked CTAs poll
     // it, and must not slow the atomics on the per-iteration counters above.

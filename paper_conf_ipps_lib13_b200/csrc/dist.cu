@@ -456,7 +456,7 @@ ag_status dist_scratch(ag_graph_s *g) {
         if ((s = dev_alloc((void **)&g->d_hub, (size_t)g->hub_cap * 8, g->device)) != AG_OK) return s;
         cudaMemset(g->d_hub, 0, (size_t)g->hub_cap * 8);
     }
-    if (!g->d_level && (s = dev_alloc((void **)&g->d_level, level_bytes((uint32_t)V), g->device)) != AG_OK) return s;
+    if (!g->d_level && (s = dev_alloc((void **)&g->d_level, V * 4 + 128, g->device)) != AG_OK) return s;
     if (!g->d_acc && (s = dev_alloc(&g->d_acc, 64, g->device)) != AG_OK) return s;
     return AG_OK;
 }

@@ -68,9 +68,6 @@ ag_status set_error(ag_status s, const char *fmt, ...);
 ag_status cuda_status(cudaError_t e, const char *what);
 ag_status dev_alloc(void **p, size_t bytes, int device);
 void dev_free(void *p, size_t bytes, int device);
-// internal level array (degree layout / distributed part): padded to whole 1024-id blocks for the BFS level
-// swizzle (traverse.cuh lvl_index)
-inline size_t level_bytes(uint32_t V) { return ((size_t)V + 1023) / 1024 * 1024 * 4 + 128; }
 bool is_device_ptr(const void *p);
 ag_status check_device(int device, int *num_sms);
 void note_launch(unsigned n);

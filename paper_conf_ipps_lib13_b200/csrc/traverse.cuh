@@ -45,14 +45,6 @@ __device__ unsigned long long g_prof[PROF_IT][PROF_CTA][6];   // [3]: adjacency 
 #define AG_PROF_MARK(it, k)
 #endif
 
-// BFS level array in the degree layout: the 32 x 32 transpose inside every 1024-id block stores the levels of
-// consecutive (= similarly hot) ids 128 B apart, so the claiming atomicMins on the hottest ids spread over 32
-// lines (L2 slices) instead of queueing on one.  The array is only written by atomics / stores and read by the
-// final pass, so nothing loses locality.  Needs the array padded to a multiple of 1024 entries.
-__host__ __device__ __forceinline__ uint32_t lvl_index(uint32_t v) {
-    return (v & ~1023u) | ((v & 31u) << 5) | ((v >> 5) & 31u);
-}
-
 template <typename Off>
 struct TravArgs {
     const Off *rp;
@@ -85,7 +77,6 @@ struct TravArgs {
     uint32_t nblocks;
     uint32_t max_iters;
     uint32_t has_hubs;
-    uint32_t lvl_swz;           // BFS, degree layout: level of v stored at lvl_index(v) (hot ids spread over lines)
     const uint2 *ulist;         // listed working set (multi-GPU SSSP): entry i = (u, dist of u); the value
                                 // travels with the entry, hub tasks carry the entry index (nullptr: off)
 };
@@ -357,7 +348,7 @@ struct Ops {
                 r[j] = 0u;
                 if ((cm >> j) & 1u) {
                     if constexpr (ORD == ORD_O) r[j] = atomicOr(a.vis + (v[j] >> 5), m);  // claim
-                    else r[j] = atomicMin(&a.level[a.lvl_swz ? lvl_index(v[j]) : v[j]], uv[j] + 1);
+                    else r[j] = atomicMin(&a.level[v[j]], uv[j] + 1);
                 }
             }
 #pragma unroll
@@ -367,7 +358,7 @@ struct Ops {
                 const bool won = ((cm >> j) & 1u) && ((ORD == ORD_O) ? !(r[j] & m) : (r[j] > nl));
                 if (won) {
                     if constexpr (ORD == ORD_O) {
-                        a.level[a.lvl_swz ? lvl_index(v[j]) : v[j]] = nl;   // m.level = level    (l.9)
+                        a.level[v[j]] = nl;                            // m.level = level    (l.9)
                         if (bm_upd) red_or(a.bm[(it + 1) % 3] + (v[j] >> 5), m);   // update vector (l.10)
                     } else {
                         red_or(a.vis + (v[j] >> 5), m);
@@ -891,7 +882,7 @@ __device__ __forceinline__ void compact_raw(const TravArgs<Off> &a, SmT &sm, uin
         __syncthreads();
         const uint32_t wbase = sm.bcast + sm.red32[1][wid], wtot = __shfl_sync(0xffffffffu, x, 31);
         warp_emit_f(q + wbase, x, c, word, w0 + (wid << 5), wtot, [&](uint32_t v) {
-            if constexpr (ALG == ALG_BFS) a.level[a.lvl_swz ? lvl_index(v) : v] = lvl;   // m.level = level (Fig. 4 l.9)
+            if constexpr (ALG == ALG_BFS) a.level[v] = lvl;   // m.level = level (Fig. 4 l.9)
         });
         __syncthreads();   // red32 / bcast reuse
     }
@@ -939,7 +930,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     // ---------------- phase 0: init (Fig. 4 lines 3-4; Fig. 8 lines 1-3) ----------------
     if (ALG == ALG_BFS) {
         for (uint32_t v = gtid; v < a.V; v += gthreads) {
-            a.level[a.lvl_swz ? lvl_index(v) : v] = (v == src) ? 0u : INF;
+            a.level[v] = (v == src) ? 0u : INF;
             if (a.parent) a.parent[v] = (v == src) ? src : INF;
         }
     } else if (ALG == ALG_CC) {   // label = own (caller) id; WS_0 = every vertex, as queue and as bitmap
@@ -1277,7 +1268,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     } else if (a.inv) {     // BFS / CC in the degree layout: gather back to caller ids
         for (uint32_t v = gtid; v < a.V; v += gthreads) {
             const uint32_t i = a.inv[v];
-            a.out_level[v] = a.level[(ALG == ALG_BFS && a.lvl_swz) ? lvl_index(i) : i];
+            a.out_level[v] = a.level[i];
             if (a.out_parent) {
                 uint32_t pp = a.parent[i];
                 a.out_parent[v] = pp == INF ? INF : a.perm[pp];
