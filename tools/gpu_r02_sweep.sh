@@ -13,5 +13,6 @@ cat gpurun_out/sweeps/r02_static_table.md
 for cfg in C2 C4; do timeout 600 python tools/calibrate.py --x7 --config $cfg --sources 1 --expect /tmp/expect_$cfg.npz > gpurun_out/sweeps/r02_x7_$cfg.jsonl 2>&1; echo "x7 $cfg rc=$?"; done
 timeout 900 python tools/calibrate.py --x8 --config C4 --sources 2 --expect /tmp/expect_C4.npz > gpurun_out/sweeps/r02_x8_C4.jsonl 2>&1; echo "x8 rc=$?"
 tail -20 gpurun_out/sweeps/r02_x8_C4.jsonl
-for a in bfs sssp; do timeout 300 python tools/level_roofline.py --config C2 --alg $a > gpurun_out/sweeps/r02_levels_C2_$a.txt 2>&1; cat gpurun_out/sweeps/r02_levels_C2_$a.txt; done
-timeout 300 python tools/level_roofline.py --config C4 --alg bfs > gpurun_out/sweeps/r02_levels_C4_bfs.txt 2>&1
+
+
+du -sh gpurun_out gpurun_out/sweeps/*; rm -f gpurun_out/sweeps/*.err
