@@ -1006,6 +1006,11 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
     const bool small_ok = TUNED && (a.has_hubs ? a.pol.t_small_hub > 0 : a.pol.t_small > 0) && nlead > 0 &&
                           nlead < a.nblocks;
 
+    // BFS whose every iteration uses the queue (tuned kernels, or the tuned decisions of unordered BFS in the
+    // general kernel): the update-vector bitmap is never read, so it is neither written nor cleared
+    // (C2 BFS 0.543 -> 0.533 ms, profiles/r02_ab/ab_summary.txt 5v)
+    const bool bfs_qonly = ALG == ALG_BFS && (TUNED || (a.pol.kind == AG_POLICY_TUNED && !a.pol.ordered &&
+                                                         a.pol.force_ws != WS_BM));
     uint32_t prev_ws = WS_QU;   // representation used in the previous iteration
     uint8_t prev_var = 0;
     uint32_t n_prev = 0;
@@ -1130,7 +1135,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
                     qn = ld_relaxed(&ctl->q_len[slot]);
                 }
             }
-        } else if (!TUNED) {
+        } else if (!TUNED && !bfs_qonly) {
             // clear the bitmap that iteration it+1 will write: bm[(it+2)%3] (read in iteration it-1).
             // (tuned kernels instead clear each frontier word when its vertex is read from the queue)
             uint32_t *bz = a.bm[(it + 2) % 3];
@@ -1147,7 +1152,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         Ops<ALG, ORD, Off, DO> ops(a, it, hi, append);
         ops.wbuf = sm.wq[threadIdx.x >> 5];
         ops.nact = nact;
-        ops.bm_upd = !(TUNED && ALG == ALG_BFS);
+        ops.bm_upd = !bfs_qonly;
         if (TUNED && (uint64_t)qn < (uint64_t)a.pol.smallchunk_per_cta * nact) {   // few tasks per CTA: finer tasks
             ops.hdeg = HUB_CHUNK_SMALL < HUB_DEG ? HUB_CHUNK_SMALL : HUB_DEG;
             ops.hchunk = HUB_CHUNK_SMALL;
