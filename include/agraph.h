@@ -207,6 +207,9 @@ ag_status ag_bfs(ag_graph g, uint32_t src, uint32_t *levels, uint32_t *parents, 
  * Unordered = Bellman-Ford-style label correcting (18.s3, 18.s5); ordered = bucketed with width
  * policy->delta (delta = 1: all pending nodes at the current minimum distance per iteration, the
  * paper's GPU Dijkstra, 28.s8; findmin by parallel reduction, 22.s11).
+ * parents = NULL (distances only, as Fig. 5 computes them) lets the tuned kernels keep a 4-byte distance per
+ * vertex instead of the packed 8-byte (distance, parent) word that keeps a parent consistent with its
+ * distance: same distances, fewer bytes per status read and per atomic.
  * Errors: as ag_bfs plus AG_ERR_NO_WEIGHTS, AG_ERR_OVERFLOW. */
 ag_status ag_sssp(ag_graph g, uint32_t src, uint32_t *dist, uint32_t *parents, const ag_policy *policy,
                   ag_run_stats *stats, void *stream);
