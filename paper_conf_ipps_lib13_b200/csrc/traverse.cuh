@@ -84,9 +84,6 @@ struct TravArgs {
 #ifndef AG_HTILE
 #define AG_HTILE BS   // hybrid mapping: queue entries per tile at most (the tile's pieces still span the CTA)
 #endif
-#ifndef AG_SMALLCHUNK_GEN
-#define AG_SMALLCHUNK_GEN 0   // finer hub tasks for small working sets also in the general kernel under the tuned policy
-#endif
 #ifndef AG_BLIND
 #define AG_BLIND 1
 #endif
@@ -1156,8 +1153,7 @@ __global__ void __launch_bounds__(BS, ALG == ALG_SSSP ? (TUNED ? AG_MINB_SSSP_T 
         ops.wbuf = sm.wq[threadIdx.x >> 5];
         ops.nact = nact;
         ops.bm_upd = !bfs_qonly;
-        if ((TUNED || (AG_SMALLCHUNK_GEN && a.pol.kind == AG_POLICY_TUNED)) &&
-            (uint64_t)qn < (uint64_t)a.pol.smallchunk_per_cta * nact) {   // few tasks per CTA: finer tasks
+        if (TUNED && (uint64_t)qn < (uint64_t)a.pol.smallchunk_per_cta * nact) {   // few tasks per CTA: finer tasks
             ops.hdeg = HUB_CHUNK_SMALL < HUB_DEG ? HUB_CHUNK_SMALL : HUB_DEG;
             ops.hchunk = HUB_CHUNK_SMALL;
         }
