@@ -160,7 +160,7 @@ typedef struct {
  * ------------------------------------------------------------------------------------------- */
 
 /* Fill *p with defaults for `device`: order UNORDERED, mapping/workset AUTO, kind TUNED,
- * T1 = 32, thread_tpb = 192, T2 = 192 x #SMs, t3_ppm = 15625, delta = 1, sample_every = 1,
+ * T1 = 32, thread_tpb = 192, T2 = 192 x #SMs, t3_ppm = 100000 (10% of V, calibrated on B200: X8), delta = 1, sample_every = 1,
  * sssp_window = AG_WINDOW_AUTO.
  * Errors: AG_ERR_INVALID_ARG (p NULL), AG_ERR_NO_DEVICE. */
 ag_status ag_policy_default(ag_policy *p, int device);

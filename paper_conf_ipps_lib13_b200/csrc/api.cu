@@ -704,7 +704,7 @@ ag_status ag_policy_default(ag_policy *p, int device) {
     p->t1_avg_degree = 32;
     p->thread_tpb = 192;
     p->t2_ws = 192ull * (uint64_t)sms;
-    p->t3_ppm = 15625;
+    p->t3_ppm = 100000;   // T3 = 10% of V: the B200 calibration (X8, profiles/sweeps/r02_x8_C4.jsonl)
     p->sample_every = 1;
     p->delta = 1;
     p->cta_group = 0;
