@@ -98,9 +98,6 @@ constexpr int EB_MAX = (AG_EB_BFS > AG_EB_SSSP) ? AG_EB_BFS : AG_EB_SSSP;
 // slot(it+2) is reset at the start of iteration it (its last reader finished at the barrier).
 // ---------------------------------------------------------------------------------------------
 constexpr int NGRP = 32;            // barrier arrival groups (hierarchical arrival)
-#ifndef AG_FENCE_ACQREL
-#define AG_FENCE_ACQREL 1
-#endif
 #ifndef AG_CTL_SPREAD
 #define AG_CTL_SPREAD 1
 #endif
@@ -305,25 +302,15 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
 // the last CTA arrives; everyone spins on that bit (measured on B200: ~1.6 us at 592 CTAs, faster
 // than a two-level tree with a separate release word).  Self-resetting across launches.
 // `first`: exactly one participating CTA passes true (default: CTA 0).
-// gpu-scope fence for the grid barrier and the hub drain: acquire-release is all they need (their writes
-// published before the arrival, the others' writes visible after the departure); __threadfence() compiles to
-// the heavier sequentially consistent MEMBAR.SC on sm_100
-__device__ __forceinline__ void fence_gpu() {
-#if AG_FENCE_ACQREL
-    asm volatile("fence.acq_rel.gpu;" ::: "memory");
-#else
-    __threadfence();
-#endif
-}
 __device__ __forceinline__ void grid_barrier(Ctl *ctl, unsigned nblocks, bool first) {
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned inc = first ? (0x80000000u - (nblocks - 1)) : 1u;
-        fence_gpu();
+        __threadfence();
         const unsigned old = atomicAdd(&ctl->bar_count, inc);
         while (((old ^ ld_relaxed(&ctl->bar_count)) & 0x80000000u) == 0) {
         }
-        fence_gpu();
+        __threadfence();
     }
     __syncthreads();
 }

@@ -84,9 +84,6 @@ struct TravArgs {
 #ifndef AG_HTILE
 #define AG_HTILE BS   // hybrid mapping: queue entries per tile at most (the tile's pieces still span the CTA)
 #endif
-#ifndef AG_DIST_L1
-#define AG_DIST_L1 1   // unordered SSSP: the expansion value read L1-cacheable (stale-high is safe)
-#endif
 #ifndef AG_BLIND
 #define AG_BLIND 1
 #endif
@@ -170,18 +167,6 @@ struct Ops {
         if constexpr (DO) return ld_relaxed(D() + u);
         else return (uint32_t)(ld_relaxed64(&a.P[u]) >> 32);
     }
-    // The value an unordered expansion starts from may be stale-high (an L1 copy): a vertex improved during
-    // this iteration was re-added to the next working set by its improver and is expanded again with the
-    // better value, so the label-correcting fixed point is unchanged.  Ordered SSSP decides bucket membership
-    // from it and reads the coherent value.
-    __device__ __forceinline__ uint32_t dist_expand(uint32_t u) const {
-        if constexpr (ORD == ORD_U && AG_DIST_L1) {
-            if constexpr (DO) return ld_keep(D() + u, pol_keep);
-            else return (uint32_t)(ld_keep(a.P + u, pol_keep) >> 32);
-        } else {
-            return dist_now(u);
-        }
-    }
     __device__ __forceinline__ uint32_t relax(uint32_t v, uint32_t nd, uint32_t u) const {
         if constexpr (DO) return atomicMin(D() + v, nd);
         else return (uint32_t)(atomicMin(&a.P[v], ((unsigned long long)nd << 32) | u) >> 32);
@@ -212,7 +197,7 @@ struct Ops {
         } else if (a.ulist) {
             // listed entry: uval (the sender's distance of u) was set by the caller; every entry expands
         } else {
-            uint32_t t = dist_expand(u);
+            uint32_t t = dist_now(u);
             uval = t;
             if constexpr (ORD == ORD_O) {
                 if ((uint64_t)t < hi) {  // in the current bucket: claim (settle) it
@@ -275,7 +260,7 @@ struct Ops {
             u = key;
             uval = (ALG == ALG_BFS) ? it
                  : (ALG == ALG_CC)  ? ld_relaxed(&a.level[u])
-                                    : dist_expand(u);
+                                    : dist_now(u);
         }
     }
 
@@ -761,7 +746,7 @@ __device__ __forceinline__ void drain_hubs(Ops<ALG, ORD, Off, DO> &ops, SmT &sm,
     uint32_t c1 = 0;                  // claimed index of the next task
     unsigned long long pre = 0ull;    // its word, fetched while the current task is expanded
     if (threadIdx.x == 0) {
-        fence_gpu();
+        __threadfence();
         atomicAdd(&ctl->stage_done[slot], 1u);
         const uint32_t c0 = atomicAdd(&ctl->hub_head[slot], 1u);
         const unsigned long long w = hub_wait(a, c0, slot, ops.nact);
