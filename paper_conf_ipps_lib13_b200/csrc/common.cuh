@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <cstddef>
 #include <type_traits>
 
 #include "agraph.h"
@@ -152,6 +153,18 @@ struct alignas(128) Ctl {
     // distance exceeds MAX_FINITE (exact, checked in-kernel), bits 8.. = max abort code seen
     unsigned int sticky;
 };
+// layout invariants: the distributed path clears the totals as one 16-byte range; with AG_CTL_SPREAD every
+// hot per-iteration counter sits on its own 128-B line (an alignas on a multi-declarator member would align
+// each declarator, which once split vexp / eexp apart)
+static_assert(offsetof(Ctl, eexp) == offsetof(Ctl, vexp) + 8, "vexp, eexp must be adjacent");
+#if AG_CTL_SPREAD
+static_assert(offsetof(Ctl, q_len) / 128 != offsetof(Ctl, tile_ctr) / 128 &&
+                  offsetof(Ctl, tile_ctr) / 128 != offsetof(Ctl, hub_tail) / 128 &&
+                  offsetof(Ctl, hub_tail) / 128 != offsetof(Ctl, hub_head) / 128 &&
+                  offsetof(Ctl, hub_head) / 128 != offsetof(Ctl, stage_done) / 128 &&
+                  offsetof(Ctl, stage_done) / 128 != offsetof(Ctl, it_edges) / 128,
+              "per-iteration control counters on separate lines");
+#endif
 
 // Policy as seen by the device (plain integers; filled from ag_policy on the host).
 struct DevPolicy {
